@@ -1,0 +1,339 @@
+"""Pins for the oracle's evaluation u*(x).
+
+Every expected value here is fixed by the paper and mathematics, not by the oracle:
+  P3  u = 1  ->  u* = 1 (the kernel integrates to 1, L202-205; pieces partition the stencil)
+  P4  polynomials of degree <= 2k (and 2k+1) are reproduced (L202-205); degree 2k+2 gives the
+      closed-form error m_{2k+2} h^{2k+2}
+  P5  separable field on a structured mesh: u*(x,y) = (K_h * f)(x), with the 1D convolution
+      computed by an exact-rational routine written here; cross-checked against SURVEY A4
+  P7  exact-rational brute force (tests/exact_siac.py) on tiny meshes
+  P8  scipy adaptive quadrature with scipy's own B-spline on single triangles
+  P9  superconvergence order >= 2k+1 on sin(2 pi x) sin(2 pi y) (L177-185, refs [8,16])
+  P10 stencil area W^2, translation invariance, grid == brute force candidate search
+"""
+import math
+import os
+from fractions import Fraction as Fr
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_0007k13_b200 import inputs
+
+from exact_siac import exact_siac, kernel_cell_polys
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def const_modes(nt, k):
+    C = np.zeros((nt, inputs.n_modes(k)))
+    C[:, 0] = math.sqrt(2.0)          # phi_00 = 1/sqrt(2)  ->  u = 1
+    return C
+
+
+# ------------------------------------------------------------------ P3 constant field
+
+@pytest.mark.parametrize("k", [1, 2, 3, 4])
+def test_constant_field_structured(oracle_mod, k):
+    V, T = inputs.structured_mesh(20)
+    h = 1 / 20
+    P = inputs.eval_points(V, T, k)[:: max(1, 3 * k)]
+    u, area = oracle_mod.oracle_eval(V, T, const_modes(len(T), k), k, h, P, return_area=True)
+    assert np.abs(u - 1).max() < 1e-13
+    assert np.abs(area - ((3 * k + 1) * h) ** 2).max() < 1e-14
+
+
+@pytest.mark.parametrize("graded", [False, True])
+def test_constant_field_unstructured(oracle_mod, graded):
+    V, T = inputs.lattice_delaunay_mesh(2000, seed=11, graded=graded)
+    k = 2
+    h = inputs.max_edge(V, T)
+    P = np.random.default_rng(0).uniform(-0.2, 1.2, (60, 2))     # also points outside [0,1)^2
+    P[:4] = [[0, 0], [1, 1], [0.5, 0], [1, 0.25]]                 # domain corners and edges
+    u, area = oracle_mod.oracle_eval(V, T, const_modes(len(T), k), k, h, P, return_area=True)
+    assert np.abs(u - 1).max() < 1e-13
+    assert np.abs(area - ((3 * k + 1) * h) ** 2).max() < 1e-13
+
+
+# ------------------------------------------------------------------ P4 polynomial reproduction
+
+def _moment(k, m):
+    """m-th moment of K from the exact coefficients and the box-sum B-spline moments."""
+    import oracle
+    c = oracle.kernel_coefficients(k)
+    mu = [oracle.bspline_moments(k, l) for l in range(m + 1)]
+    return sum(cg * sum(math.comb(m, l) * Fr(g - k) ** (m - l) * mu[l] for l in range(m + 1))
+               for g, cg in enumerate(c))
+
+
+@pytest.mark.parametrize("k", [1, 2])
+def test_monomial_reproduction_and_negative_control(oracle_mod, k):
+    """(K_h x K_h) * (y1^a y2^b) = prod over axes of sum_l C(n,l) x^(n-l) h^l m_l.
+    With m_1..m_{2k+1} = 0 this is x1^a x2^b for a, b <= 2k+1 and picks up exactly
+    m_{2k+2} h^{2k+2} at degree 2k+2.  Non-periodic mesh, interior points."""
+    V, T = inputs.lattice_delaunay_mesh(600, seed=4)
+    h = 0.04
+    W = (3 * k + 1) * h
+    rng = np.random.default_rng(1)
+    P = rng.uniform(W / 2 + 0.01, 1 - W / 2 - 0.01, (12, 2))
+    d = 2 * k + 2
+    for a, b in [(0, 0), (1, 0), (0, 2 * k), (2 * k, 2 * k), (2 * k + 1, 1), (d, 0), (d, 1), (2, d)]:
+        A = np.zeros((d + 1, d + 1))
+        A[a, b] = 1.0
+        u = oracle_mod.oracle_eval(V, T, A, k, h, P, periodic=0, field_mode=1, field_deg=d)
+
+        def conv(x, n):
+            return sum(math.comb(n, l) * x ** (n - l) * h ** l * float(_moment(k, l)) for l in range(n + 1))
+
+        expect = np.array([conv(x1, a) * conv(x2, b) for x1, x2 in P])
+        assert np.abs(u - expect).max() < 1e-13, (a, b)
+        if a <= 2 * k + 1 and b <= 2 * k + 1:
+            assert np.abs(u - P[:, 0] ** a * P[:, 1] ** b).max() < 1e-13
+        else:
+            assert np.abs(u - P[:, 0] ** a * P[:, 1] ** b).max() > 1e-3 * h ** d
+
+
+@pytest.mark.parametrize("k", [1, 2, 3])
+def test_dg_polynomial_reproduction(oracle_mod, k):
+    """u_h = a global polynomial of degree <= k (exactly representable) -> u* = u."""
+    V, T = inputs.lattice_delaunay_mesh(800, seed=5)
+    f = lambda x, y: 0.2 + (x - 0.3 * y) ** k - 0.7 * x * y ** (k - 1)  # noqa: E731
+    C = inputs.project(V, T, k, f)
+    h = 0.03
+    W = (3 * k + 1) * h
+    P = np.random.default_rng(2).uniform(W / 2 + 0.01, 1 - W / 2 - 0.01, (10, 2))
+    u = oracle_mod.oracle_eval(V, T, C, k, h, P, periodic=0)
+    assert np.abs(u - f(P[:, 0], P[:, 1])).max() < 1e-13
+
+
+# ------------------------------------------------------------------ P5 separable closed form
+
+LEG = [[Fr(1)], [Fr(0), Fr(1)], [Fr(-1, 2), Fr(0), Fr(3, 2)], [Fr(0), Fr(-3, 2), Fr(0), Fr(5, 2)]]
+
+
+def _poly_shift_scale(coefs, a, b):
+    """p(a + b t) as coefficients in t."""
+    out = [Fr(0)] * len(coefs)
+    for n, c in enumerate(coefs):
+        for j in range(n + 1):
+            out[j] += c * math.comb(n, j) * a ** (n - j) * b ** j
+    return out
+
+
+def exact_1d(k, N, modes, x):
+    """(1/h) int K((y-x)/h) f(y) dy on the periodic grid, exactly (test-local routine)."""
+    import oracle
+    h = Fr(1, N)
+    x = Fr(x)
+    kp = kernel_cell_polys(k, oracle.kernel_coefficients(k))
+    lo = Fr(-(3 * k + 1), 2)
+    tot = Fr(0)
+    for m in range(3 * k + 1):
+        A, B = x + h * (lo + m), x + h * (lo + m + 1)        # kernel cell in y
+        for s in (-1, 0, 1):
+            for i in range(N):
+                c0, c1 = i * h + s, (i + 1) * h + s          # image of mesh cell i
+                a, b = max(A, c0), min(B, c1)
+                if a >= b:
+                    continue
+                # f on this cell as a polynomial in y: xi = 2(y - s - (i+1/2)h)/h
+                fy = [Fr(0)] * (k + 1)
+                for j, amp in enumerate(modes[i]):
+                    pj = _poly_shift_scale(LEG[j], -2 * (s + (i + Fr(1, 2)) * h) / h, 2 / h)
+                    for n, c in enumerate(pj):
+                        fy[n] += Fr(amp) * c
+                ky = _poly_shift_scale(kp[m], -x / h, 1 / h)    # K_m((y - x)/h)
+                prod = [Fr(0)] * (len(fy) + len(ky) - 1)
+                for p1, c1_ in enumerate(fy):
+                    for p2, c2_ in enumerate(ky):
+                        prod[p1 + p2] += c1_ * c2_
+                tot += sum(c * (b ** (n + 1) - a ** (n + 1)) / (n + 1) for n, c in enumerate(prod))
+    return tot / h
+
+
+def _gold_1d():
+    rows = []
+    for line in open(os.path.join(GOLD, "siac_1d_values.txt")):
+        line = line.strip()
+        if line and not line.startswith("#"):
+            k, N, x, v = line.split()
+            rows.append((int(k), int(N), Fr(x), Fr(v)))
+    return rows
+
+
+MODES_1D = {1: [(1, 0), (0, 1), (-1, Fr(1, 2)), (2, -1)],
+            2: [(1, 0, 0), (0, 1, 0), (0, 0, 1), (1, -1, 1), (-1, 0, 2), (2, 1, 0), (0, -2, 1), (1, 1, 1)]}
+
+
+def test_exact_1d_routine_matches_survey_values():
+    for k, N, x, v in _gold_1d():
+        assert exact_1d(k, N, MODES_1D[k], x) == v
+
+
+@pytest.mark.parametrize("k", [1, 2])
+def test_separable_lift_2d(oracle_mod, k):
+    """u_h(x, y) = f(x) on the periodic N x N '/' mesh -> u*(x, y) = f*(x) for all y (P5)."""
+    N = {1: 4, 2: 8}[k]
+    modes = MODES_1D[k]
+    V, T = inputs.structured_mesh(N)
+
+    def f(X, Y):
+        i = np.clip(np.floor(X * N).astype(int), 0, N - 1)
+        xi = 2 * (X - (i + 0.5) / N) * N
+        out = np.zeros_like(X)
+        for j in range(k + 1):
+            amp = np.array([float(modes[ii][j]) for ii in range(N)])[i]
+            out += amp * np.polynomial.legendre.legval(xi, [0] * j + [1])
+        return out
+
+    C = inputs.project(V, T, k, f)
+    xs = [x for kk, NN, x, _ in _gold_1d() if kk == k]
+    ys = [0.0, 0.1234, 0.5, 0.87]
+    P = np.array([[float(x), y] for x in xs for y in ys])
+    u = oracle_mod.oracle_eval(V, T, C, k, 1 / N, P)
+    expect = np.array([float(exact_1d(k, N, modes, x)) for x in xs for _ in ys])
+    assert np.abs(u - expect).max() < 1e-13
+
+
+# ------------------------------------------------------------------ P7 exact rational brute force
+
+def _tiny_mesh():
+    """3 x 3 periodic '/' mesh with the 4 interior vertices moved by rational offsets."""
+    n = 3
+    V = [[Fr(i, n), Fr(j, n)] for j in range(n + 1) for i in range(n + 1)]
+    moves = {(1, 1): (Fr(1, 17), Fr(-1, 23)), (2, 1): (Fr(-1, 19), Fr(1, 29)),
+             (1, 2): (Fr(1, 31), Fr(1, 13)), (2, 2): (Fr(-1, 11), Fr(-1, 37))}
+    for (i, j), (dx, dy) in moves.items():
+        V[j * (n + 1) + i][0] += dx
+        V[j * (n + 1) + i][1] += dy
+    _, T = inputs.structured_mesh(n)
+    return V, T.tolist()
+
+
+@pytest.mark.parametrize("k,h,pts", [
+    (1, Fr(1, 5), [(Fr(1, 7), Fr(2, 9)), (Fr(19, 20), Fr(1, 30)), (Fr(1, 2), Fr(1, 2))]),
+    (2, Fr(1, 8), [(Fr(3, 7), Fr(5, 6)), (Fr(1, 40), Fr(97, 100))]),
+])
+def test_exact_rational_brute_force(oracle_mod, k, h, pts):
+    import oracle
+    Vq, Tl = _tiny_mesh()
+    rng = np.random.default_rng(7 + k)
+    mons = [(a, b) for a in range(k + 1) for b in range(k + 1 - a)]
+    fields = [{m: Fr(int(rng.integers(-9, 10)), int(rng.integers(1, 7))) for m in mons} for _ in Tl]
+    coeffs = oracle.kernel_coefficients(k)
+    exact = [exact_siac(Vq, Tl, fields, k, h, coeffs, x) for x in pts]
+
+    V = np.array([[float(a), float(b)] for a, b in Vq])
+    T = np.array(Tl, dtype=np.int32)
+    cf = np.array([[float(fl[m]) for m in mons] for fl in fields])
+
+    def f(X, Y):
+        return sum(cf[:, i][:, None] * X ** a * Y ** b for i, (a, b) in enumerate(mons))
+
+    C = inputs.project(V, T, k, f)
+    u = oracle_mod.oracle_eval(V, T, C, k, float(h), np.array([[float(a), float(b)] for a, b in pts]))
+    ex = np.array([float(e) for e in exact])
+    assert np.abs(u - ex).max() < 1e-13 * max(1.0, np.abs(ex).max())
+
+
+# ------------------------------------------------------------------ P8 adaptive quadrature
+
+def test_adaptive_quadrature_single_triangles(oracle_mod):
+    """scipy.integrate.quad (nested, with the kernel breakpoints) and scipy's BSpline on
+    single triangles in the stencil, one point each."""
+    from scipy.integrate import quad
+    from scipy.interpolate import BSpline
+    import oracle
+
+    k, h = 2, 0.1
+    c = [float(v) for v in oracle.kernel_coefficients(k)]
+    psi = BSpline.basis_element(np.arange(k + 2) - (k + 1) / 2, extrapolate=False)
+
+    def K(t):
+        v = sum(cg * np.nan_to_num(psi(t - (g - k))) for g, cg in enumerate(c))
+        return float(v)
+
+    rng = np.random.default_rng(3)
+    x = np.array([0.5, 0.5])
+    breaks = x[0] + h * (np.arange(3 * k + 2) - (3 * k + 1) / 2)
+    for trial in range(3):
+        tri = x + rng.uniform(-0.3, 0.3, (3, 2))
+        V = tri
+        T = np.array([[0, 1, 2]], dtype=np.int32)
+        fcoef = rng.uniform(-1, 1, 3)
+        f = lambda X, Y: fcoef[0] + fcoef[1] * X + fcoef[2] * X * Y  # noqa: E731
+        C = inputs.project(V, T, k, f)
+        u = oracle_mod.oracle_eval(V, T, C, k, h, x[None, :], periodic=0)[0]
+        # reference: integrate over the triangle, x-slices between sorted vertices
+        order = np.argsort(tri[:, 0])
+        A, B, Cc = tri[order]
+
+        def yr(xx):
+            ys = []
+            for P1, P2 in ((A, B), (B, Cc), (A, Cc)):
+                if min(P1[0], P2[0]) <= xx <= max(P1[0], P2[0]) and P1[0] != P2[0]:
+                    ys.append(P1[1] + (xx - P1[0]) / (P2[0] - P1[0]) * (P2[1] - P1[1]))
+            return min(ys), max(ys)
+
+        def inner(xx):
+            lo, hi = yr(xx)
+            pts = [b for b in breaks if lo < b < hi]
+            return quad(lambda yy: K((yy - x[1]) / h) * f(xx, yy), lo, hi, points=pts or None,
+                        epsabs=1e-14, epsrel=1e-12, limit=200)[0] * K((xx - x[0]) / h)
+
+        ref = 0.0
+        for a, b in ((A[0], B[0]), (B[0], Cc[0])):
+            if b > a:
+                pts = [q for q in breaks if a < q < b]
+                ref += quad(inner, a, b, points=pts or None, epsabs=1e-13, epsrel=1e-11, limit=200)[0]
+        ref /= h * h
+        assert u == pytest.approx(ref, abs=1e-8)
+
+
+# ------------------------------------------------------------------ P9 superconvergence
+
+@pytest.mark.parametrize("k,Ns", [(1, (10, 20, 40, 80)), (2, (10, 20, 40)), (3, (10, 20, 40))])
+def test_superconvergence_order(oracle_mod, k, Ns):
+    """Filtered error at the evaluation points decays at order >= 2k+1 (refs [8], [16];
+    SURVEY Q17) on u = sin(2 pi x) sin(2 pi y), structured periodic meshes, h = 1/N."""
+    errs = []
+    rng = np.random.default_rng(9)
+    for N in Ns:
+        V, T = inputs.structured_mesh(N)
+        C = inputs.project(V, T, k, inputs.sinsin, n_quad=k + 8)
+        sel = rng.choice(len(T), size=min(len(T), 300), replace=False)
+        P = inputs.eval_points(V, T[sel], k)
+        u = oracle_mod.oracle_eval(V, T, C, k, 1 / N, P)
+        errs.append(np.abs(u - inputs.sinsin(P[:, 0], P[:, 1])).max())
+    rates = [math.log2(errs[i] / errs[i + 1]) for i in range(len(errs) - 1)]
+    assert min(rates) >= 2 * k + 1 - 0.2, (errs, rates)
+
+
+# ------------------------------------------------------------------ P10 invariants
+
+def test_translation_invariance_structured(oracle_mod):
+    """Translating the field by whole mesh cells (with wrap) translates u* (P10)."""
+    N, k = 8, 2
+    V, T = inputs.structured_mesh(N)
+    C = inputs.random_modes(len(T), k, seed=3)
+    a, b = 3, 5
+    C2 = np.empty_like(C)
+    for j in range(N):
+        for i in range(N):
+            src = 2 * (j * N + i)
+            dst = 2 * (((j + b) % N) * N + (i + a) % N)
+            C2[dst:dst + 2] = C[src:src + 2]
+    P = np.random.default_rng(4).uniform(0, 1, (20, 2))
+    P2 = (P + np.array([a / N, b / N])) % 1.0
+    h = 1 / N
+    u1 = oracle_mod.oracle_eval(V, T, C, k, h, P)
+    u2 = oracle_mod.oracle_eval(V, T, C2, k, h, P2)
+    assert np.abs(u1 - u2).max() < 1e-13
+
+
+def test_grid_equals_brute_force(oracle_mod):
+    w = inputs.make_config(2, field_kind="random")
+    P = w.points[::997]
+    u1 = oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, P, use_grid=True)
+    u2 = oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, P, use_grid=False)
+    assert np.abs(u1 - u2).max() < 1e-13 * np.abs(u2).max()
