@@ -1,0 +1,314 @@
+#!/usr/bin/env python3
+"""bench.py -- filtered quadrature points/s (FP64) of the B200 SIAC path.
+
+Contract (driver): `python bench.py --gpus N --steps K --warmup W` (torchrun for N > 1)
+prints ONE JSON line on rank 0.  A step = one siac_eval_async over every evaluation point of
+the workload (all §8(a) rows: point keys + sort, candidate search, clipping, fan
+triangulation, quadrature, per-point reduction), inputs resident in HBM.  Default workload:
+BASELINE.json config 5 (Delaunay ~1M triangles, P3, 12 points/element = 12.6M points), the
+configuration the metric is quoted on at 1/2/4/8 GPUs; it fits one GPU.
+
+`--impl reference` times the oracle (the CPU reference arm of this tier) on a bounded
+sample of the same workload.
+"""
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+# quadrature points per sub-triangle and FP64 flops per quadrature point:
+# F_qp = 2 (n_b + 2k + 8)  (affine map 4, two degree-k Horner 2k, frame offsets 2,
+# bivariate Horner n_b - 1, product/weight/accumulate 3; an FMA counts 2 flops)
+NQ = {1: 4, 2: 12, 3: 19, 4: 33}
+
+
+def flops_per_subtri(k):
+    nb = (k + 1) * (k + 2) // 2
+    return NQ[k] * 2 * (nb + 2 * k + 8)
+
+
+def fp64_peak_derived(sm_mhz=1965.0, sms=148):
+    """148 SMs x 64 FP64 FMA lanes/clk x 2 flops x clock (B200 datasheet 37 TFLOP/s class)."""
+    return sms * 64 * 2 * sm_mhz * 1e6 / 1e12
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = "index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, device_index=0):
+        self.dev = device_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except (FileNotFoundError, OSError):
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax.append(float(f[2]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(smax), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def load_workload(cfg, field="sinsin"):
+    from paper_conf_sc_0007k13_b200 import inputs
+    return inputs.make_config(cfg, field_kind=field)
+
+
+def workload_desc(w, cfg):
+    return {"workload": f"cfg{cfg}: {w.meta['desc']}", "n_triangles": int(len(w.T)), "n_points": int(w.n_points),
+            "k": w.k, "h": w.h, "periodic": "xy", "seed": w.seed, "field": "sin(2pi x) sin(2pi y), L2-projected",
+            "points": "degree-2k symmetric-rule nodes per element"}
+
+
+def cpu_baseline(w, sample_stride, nthreads=0):
+    """The oracle as it stands, on a deterministic stride sample of the workload's points."""
+    import oracle
+    P = w.points[::sample_stride]
+    t0 = time.perf_counter()
+    oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P, nthreads=nthreads)
+    dt = time.perf_counter() - t0
+    return {"value": len(P) / dt, "unit": "points/s", "cores": nthreads or oracle.omp_threads(), "kind": "oracle",
+            "sample": f"every {sample_stride}th evaluation point ({len(P)} points), {dt:.1f} s"}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    w = load_workload(args.config)
+    import oracle
+    stride = max(1, w.n_points // args.ref_points)
+    P = w.points[::stride]
+    for _ in range(args.warmup):
+        oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P[:64])
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    val = len(P) * args.steps / tot
+    line = {"metric": "filtered quadrature points/sec (FP64)", "impl": "reference", "value": val,
+            "unit": "points/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * tot / args.steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": dict(workload_desc(w, args.config), sample=f"every {stride}th point ({len(P)} points) per step"),
+            "cpu_baseline": {"value": val, "unit": "points/s", "cores": oracle.omp_threads(), "kind": "oracle",
+                             "sample": f"every {stride}th evaluation point ({len(P)} points) per step"},
+            "e2e": {"value": val, "unit": "points/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_siac(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_0007k13_b200 import siac
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+
+    w = load_workload(args.config)
+    k = w.k
+    if world > 1:
+        from paper_conf_sc_0007k13_b200 import dist as sdist
+        part = sdist.partition(w, world)
+        sub = sdist.local_problem(w, part, rank)
+        V, T, C, P_local = sub["V"], sub["T"], sub["C"], sub["points"]
+    else:
+        part = None
+        V, T, C, P_local = w.V, w.T, w.C, w.points
+    ctx = siac.create(V, T, C, k, w.h, periodic=3, device=local)
+    n_local = len(P_local)
+    d_pts = torch.from_numpy(np.ascontiguousarray(P_local)).to(dev)
+    d_out = torch.empty(max(n_local, 1), dtype=torch.float64, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    # geometry counts (untimed): the algorithmic flop count of the quadrature
+    ctx.set_counting(True)
+    ctx.eval_async(d_pts, d_out, stream)
+    stats = ctx.stats()
+    ctx.set_counting(False)
+    subtris = stats["subtris"]
+    if world > 1:
+        t = torch.tensor([subtris, stats["pairs"], stats["pieces"], stats["candidates"]], dtype=torch.int64, device=dev)
+        dist.all_reduce(t)
+        subtris, pairs, pieces, cands = [int(x) for x in t.tolist()]
+    else:
+        pairs, pieces, cands = stats["pairs"], stats["pieces"], stats["candidates"]
+    flops_step = subtris * flops_per_subtri(k)           # whole job, per step
+
+    gathered = None
+    if world > 1:
+        nmax = part["max_count"]
+        send = torch.zeros(nmax, dtype=torch.float64, device=dev)
+        gathered = torch.empty(world * nmax, dtype=torch.float64, device=dev)
+
+    def step():
+        ctx.eval_async(d_pts, d_out, stream)
+        if world > 1:
+            send[:n_local].copy_(d_out[:n_local])
+            dist.all_gather_into_tensor(gathered, send)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ctx.timing()                       # discard
+    ctx.set_timing(True)
+    clocks = ClockSampler(local)
+    clocks.start()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    ms_total = e0.elapsed_time(e1)
+    kern_ms, kern_n = ctx.timing()
+    ctx.set_timing(False)
+    if world > 1:
+        t = torch.tensor([ms_total, kern_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total, kern_ms = t.tolist()
+    ms_step = ms_total / args.steps
+    value = w.n_points / (ms_step * 1e-3)
+
+    # end-to-end through the public host-buffer API (siac_eval): H2D of the points from pinned
+    # memory, evaluation, D2H of the values, every step
+    h_pts = torch.from_numpy(np.ascontiguousarray(P_local)).pin_memory()
+    h_out = torch.empty(max(n_local, 1), dtype=torch.float64).pin_memory()
+    hp, ho = h_pts.numpy(), h_out.numpy()
+    ctx.eval_into(hp, ho)
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(args.e2e_steps):
+        ctx.eval_into(hp, ho)
+    e2e_s = time.perf_counter() - t0
+    if world > 1:
+        t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_s = t.item()
+    e2e_val = w.n_points / (e2e_s / args.e2e_steps)
+
+    peak_meas = siac.probe_fp64(local)
+    line = None
+    if rank == 0:
+        kern_avg_s = (kern_ms / max(kern_n, 1)) * 1e-3
+        achieved = flops_step / max(world, 1) / kern_avg_s / 1e12 if kern_avg_s > 0 else None
+        peak = fp64_peak_derived()
+        cfgd = workload_desc(w, args.config)
+        cfgd.update({"parallelism": f"spatial point tiles x{world}" if world > 1 else "single GPU",
+                     "l2": "inputs larger than L2 (points %.0f MB + triangle records %.0f MB > 126 MB)"
+                           % (w.n_points * 16 / 1e6, len(w.T) * 22 * 8 / 1e6),
+                     "counts": {"candidates": cands, "pairs": pairs, "pieces": pieces, "subtris": subtris},
+                     "flops_per_subtri": flops_per_subtri(k)})
+        line = {"metric": "filtered quadrature points/sec (FP64)", "value": value, "unit": "points/s",
+                "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic", "config": cfgd,
+                "roofline": {"bound": "alu", "kernel": "k_eval", "achieved": achieved, "peak": peak,
+                             "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None, "traffic": None,
+                             "peak_note": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1965 MHz",
+                             "measured_dfma_peak": peak_meas,
+                             "frac_of_measured": (achieved / peak_meas) if achieved else None,
+                             "kernel_share_of_step": (kern_ms / kern_n) / ms_step if kern_n else None,
+                             "algorithmic_flops_per_step": flops_step},
+                "e2e": {"value": e2e_val, "unit": "points/s", "h2d_bytes_per_step": int(w.n_points * 16),
+                        "d2h_bytes_per_step": int(w.n_points * 8)},
+                "gpu_launches": 2 * args.steps,
+                "gpu_launches_note": "per step: k_point_keys + k_eval (ours) + CUB radix-sort kernels (library)",
+                "clocks": clk}
+    if rank == 0 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(w, max(1, w.n_points // args.ref_points))
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    ctx.destroy()
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=5)
+    ap.add_argument("--impl", default="siac", choices=["siac", "reference"])
+    ap.add_argument("--ref-points", type=int, default=4000, help="oracle sample size (points)")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_siac(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,162 @@
+/*
+ * siac.h -- C ABI of the B200 SIAC post-processor (libsiac_b200.so).
+ *
+ * What it computes (King & Kirby, SC'13; /root/reference/PAPER.md):
+ *   For every evaluation point x, the SIAC-filtered value of a 2D dG solution u_h,
+ *       u*(x) = (1/h^2) \int\int K((y1-x1)/h) K((y2-x2)/h) u_h(y) dy          (Eq. (1))
+ *   K(t) = sum_{g=0}^{2k} c_g psi_{k+1}(t - x_g), x_g = -k + g, psi_{k+1} the centred
+ *   B-spline of order k+1 (L196-208); Supp K = (3k+1) (L250-254).  Each triangle the
+ *   stencil touches is split along the kernel breaklines into pieces on which the integrand
+ *   is polynomial, the pieces are triangulated and integrated exactly by Gauss quadrature
+ *   (Eq. (2); Sutherland-Hodgman clipping, Alg. 1).  Periodic axes
+ *   wrap the stencil around the domain (L280-282).
+ *
+ * Conventions
+ *   - All functions are extern "C", never throw, and return siac_status (0 = OK).
+ *   - Precision: IEEE FP64 throughout; results differ from the exact integral only by
+ *     rounding (any summation order).
+ *   - Ownership: siac_create deep-copies every input (the caller may free them on return);
+ *     the context owns all device memory until siac_destroy.  siac_eval / siac_eval_async
+ *     write n_points doubles to caller-owned memory, in input order.
+ *   - Errors: on failure a message is available from siac_last_error(ctx) (ctx may be NULL
+ *     for errors of siac_create; the message is then thread-local).  No partial results are
+ *     promised on failure.  CUDA errors are reported as SIAC_ECUDA with cudaGetErrorString.
+ *   - Thread safety: one host thread at a time per context, and at most one evaluation in
+ *     flight per context (scratch buffers are per context).  Different contexts on
+ *     different devices may be used concurrently (one per rank in multi-GPU runs).
+ *   - No CPU fallback: every evaluation step runs in CUDA kernels on the context's device.
+ */
+#ifndef SIAC_H
+#define SIAC_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct siac_ctx siac_ctx;
+
+typedef enum {
+    SIAC_OK = 0,
+    SIAC_EINVAL = -1,     /* invalid argument (message says which) */
+    SIAC_ENOMEM = -2,     /* host or device allocation failed */
+    SIAC_ECUDA = -3,      /* a CUDA runtime call or kernel failed */
+    SIAC_EDEVICE = -4,    /* no usable sm_100 device at params->device */
+    SIAC_EINTERNAL = -5   /* internal invariant violated (bug) */
+} siac_status;
+
+/* Periodicity bits (all the paper's tests are periodic, L715). */
+#define SIAC_PERIODIC_X 1
+#define SIAC_PERIODIC_Y 2
+
+typedef struct {
+    int32_t k;          /* dG degree = B-spline degree; 1..4 (paper tested 1..3, L716-718) */
+    double  h;          /* kernel scaling > 0; the paper uses the longest edge s (L430, L440) */
+    int32_t periodic;   /* SIAC_PERIODIC_X | SIAC_PERIODIC_Y; non-periodic axes use zero
+                           extension outside the mesh */
+    double  domain[4];  /* x0, y0, x1, y1; the paper uses [0,1]^2 (L428) */
+    int32_t device;     /* CUDA device ordinal */
+    double  cell_factor;/* binning cell size / h; 0 -> default 0.5 (paper c_e = s/2, L505-508) */
+} siac_params;
+
+typedef struct {        /* geometry counts of the last evaluation (see siac_set_counting) */
+    int64_t n_points;
+    int64_t candidates; /* (point, triangle image) bounding-box tests */
+    int64_t pairs;      /* (point, triangle image) pairs whose boxes overlap */
+    int64_t pieces;     /* non-empty clipped polygons (triangle image ∩ kernel cell) */
+    int64_t subtris;    /* fan sub-triangles integrated = sum over pieces of (vertices - 2) */
+} siac_counters;
+
+/*
+ * siac_create -- ingest a mesh and its dG modes onto the device and build the spatial index.
+ *   vertices_xy  host, n_vertices x 2 doubles, row-major (x, y).  On periodic axes every
+ *                vertex must lie in [x0, x1] (tolerance 1e-9 of the extent).
+ *   triangles    host, n_triangles x 3 int32, 0-based vertex indices; any orientation.
+ *   coeffs       host, n_triangles x (k+1)(k+2)/2 doubles: coefficients of the orthonormal
+ *                Dubiner basis on the reference triangle {xi, eta >= -1, xi + eta <= 0},
+ *                triangle vertices 0, 1, 2 mapped to (-1,-1), (1,-1), (-1,1);
+ *                phi_pq = sqrt((2p+1)(p+q+1)/2) P_p(a) ((1-eta)/2)^p P_q^(2p+1,0)(eta),
+ *                a = 2(1+xi)/(1-eta) - 1; modes ordered by p+q, then q (PAPER.md L209-212,
+ *                L716-718: "an array of the polynomial modes"; basis per SURVEY Q8).
+ *   params       see siac_params.
+ *   *out         receives the context (NULL on failure).
+ * Errors: SIAC_EINVAL for k outside 1..4, h <= 0 or non-finite, (3k+1)h larger than a
+ *   periodic extent, an empty or inverted domain, out-of-range indices, zero-area triangles,
+ *   non-finite coordinates or coefficients, vertices outside a periodic axis; SIAC_EDEVICE,
+ *   SIAC_ENOMEM, SIAC_ECUDA.  n_triangles == 0 is allowed (every value is then 0).
+ */
+siac_status siac_create(siac_ctx **out,
+                        const double *vertices_xy, int64_t n_vertices,
+                        const int32_t *triangles, int64_t n_triangles,
+                        const double *coeffs, const siac_params *params);
+
+/*
+ * siac_eval -- blocking evaluation with HOST buffers.
+ *   points_xy   host, n_points x 2 doubles (x, y); any location (periodic axes wrap).
+ *   values_out  host, n_points doubles, written in input order.
+ * Includes the host->device copy of the points and the device->host copy of the values.
+ * n_points == 0 is a no-op returning SIAC_OK.
+ */
+siac_status siac_eval(siac_ctx *ctx, const double *points_xy, int64_t n_points, double *values_out);
+
+/*
+ * siac_eval_async -- stream-ordered evaluation with DEVICE buffers on the context's device.
+ *   d_points_xy   device, n_points x 2 doubles; must stay valid until the stream passes.
+ *   d_values_out  device, n_points doubles (input order).
+ *   cuda_stream   a cudaStream_t (NULL = legacy default stream).
+ * Returns after enqueueing (the first call for a given size may allocate scratch memory,
+ * which synchronises the device).
+ */
+siac_status siac_eval_async(siac_ctx *ctx, const double *d_points_xy, int64_t n_points,
+                            double *d_values_out, void *cuda_stream);
+
+/* Enable (1) / disable (0) geometry counting in later evaluations (adds atomics; off by default). */
+siac_status siac_set_counting(siac_ctx *ctx, int32_t enable);
+
+/* Counters of the last evaluation run with counting enabled (synchronises the device). */
+siac_status siac_stats(siac_ctx *ctx, siac_counters *out);
+
+/* Enable (1) / disable (0) CUDA-event timing of the main evaluation kernel (k_eval) on the
+ * evaluation stream.  While enabled, every evaluation records one event pair around it. */
+siac_status siac_set_timing(siac_ctx *ctx, int32_t enable);
+
+/* Sum of the main-kernel durations (ms) and number of timed launches since the last call;
+ * synchronises on the recorded events and resets the accumulator. */
+siac_status siac_timing(siac_ctx *ctx, double *kernel_ms_total, int64_t *n_launches);
+
+/* FP64 FMA throughput probe on `device`: a DFMA-chain kernel filling every SM; writes the
+ * achieved TFLOP/s (2 flops per DFMA) to *tflops.  Used as the measured roofline peak. */
+siac_status siac_probe_fp64(int32_t device, double *tflops);
+
+/* Mesh-side info: n_triangles, binning grid size, cells, max bbox extents. */
+siac_status siac_info(const siac_ctx *ctx, int64_t *n_triangles, int32_t *grid_nx, int32_t *grid_ny,
+                      double *cell_w, double *cell_h);
+
+/* Host-side exact constants (diagnostics and CPU tests; no device needed):
+ *   cell_table    (3k+1) x (k+1) doubles: K on kernel cell i as sum_m T[i][m] tau^m,
+ *                 tau = t - (t_i + 1/2), t_i = -(3k+1)/2 + i;
+ *   basis_matrix  nb x nb doubles, nb = (k+1)(k+2)/2: row i = Dubiner mode i written in the
+ *                 centred monomials rho^a sigma^b (rho = 3r-1, sigma = 3s-1), columns in the
+ *                 device Horner order (a = k..0, b = 0..k-a).
+ * Either pointer may be NULL. */
+siac_status siac_host_tables(int32_t k, double *cell_table, double *basis_matrix);
+
+/* Copy the first n device triangle records (record layout of csrc/siac_device.cuh, in
+ * binning order) to host memory `out` (n * record_doubles); *record_doubles receives the
+ * record length.  Diagnostics only. */
+siac_status siac_debug_records(siac_ctx *ctx, int64_t n, double *out, int32_t *record_doubles);
+
+/* Free everything the context owns.  NULL-safe. */
+void siac_destroy(siac_ctx *ctx);
+
+/* Last error message for ctx (or the calling thread's last siac_create error if ctx is NULL). */
+const char *siac_last_error(const siac_ctx *ctx);
+
+/* Library version string. */
+const char *siac_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SIAC_H */

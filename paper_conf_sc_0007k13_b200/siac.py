@@ -1,0 +1,248 @@
+"""Thin Python binding of libsiac_b200.so (include/siac.h) -- argument marshalling only.
+
+Every step of the path runs in the CUDA library; there is no CPU fallback.  If the shared
+library is missing or fails to load, importing this module's functions raises.
+
+    ctx = siac.create(V, T, C, k=3, h=0.01)          # siac_create
+    vals = ctx.eval(points)                           # siac_eval (host buffers)
+    ctx.eval_async(d_points, d_out, stream)           # siac_eval_async (device pointers / tensors)
+    ctx.set_counting(True); ctx.stats()               # siac_set_counting / siac_stats
+    ctx.destroy()                                     # siac_destroy
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsiac_b200.so")
+SOURCES = [os.path.join(_HERE, "csrc", f) for f in ("siac.cu", "siac_device.cuh", "siac_math.cpp", "siac_math.h",
+                                                    "siac_quadrature.h")]
+SOURCES.append(os.path.join(os.path.dirname(_HERE), "include", "siac.h"))
+
+NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
+              "-Xcompiler", "-fPIC", "-shared"]
+
+SIAC_PERIODIC_X = 1
+SIAC_PERIODIC_Y = 2
+
+
+def build(force: bool = False, verbose: bool = False) -> str:
+    """Compile csrc/siac.cu for sm_100a into paper_conf_sc_0007k13_b200/libsiac_b200.so."""
+    stale = force or not os.path.exists(LIB_PATH) or any(
+        os.path.getmtime(LIB_PATH) < os.path.getmtime(s) for s in SOURCES)
+    if stale:
+        nvcc = os.environ.get("NVCC", "nvcc")
+        obj = os.path.join(_HERE, "csrc", "siac_math.o")
+        subprocess.check_call(["g++", "-O2", "-std=c++17", "-fPIC", "-c", "-o", obj,
+                               os.path.join(_HERE, "csrc", "siac_math.cpp")])
+        cmd = [nvcc] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + \
+              ["-o", LIB_PATH + ".tmp", os.path.join(_HERE, "csrc", "siac.cu"), obj]
+        subprocess.check_call(cmd)
+        os.replace(LIB_PATH + ".tmp", LIB_PATH)
+    return LIB_PATH
+
+
+class SiacError(RuntimeError):
+    pass
+
+
+class _Params(ctypes.Structure):
+    _fields_ = [("k", ctypes.c_int32), ("h", ctypes.c_double), ("periodic", ctypes.c_int32),
+                ("domain", ctypes.c_double * 4), ("device", ctypes.c_int32), ("cell_factor", ctypes.c_double)]
+
+
+class _Counters(ctypes.Structure):
+    _fields_ = [("n_points", ctypes.c_int64), ("candidates", ctypes.c_int64), ("pairs", ctypes.c_int64),
+                ("pieces", ctypes.c_int64), ("subtris", ctypes.c_int64)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libsiac_b200.so (raises if it is missing: no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} not built; run __graft_entry__.build() (no CPU fallback exists)")
+        L = ctypes.CDLL(LIB_PATH)
+        vp, D, I64, I32 = ctypes.c_void_p, ctypes.POINTER(ctypes.c_double), ctypes.c_int64, ctypes.c_int32
+        L.siac_create.restype = ctypes.c_int
+        L.siac_create.argtypes = [ctypes.POINTER(vp), D, I64, ctypes.POINTER(ctypes.c_int32), I64, D,
+                                  ctypes.POINTER(_Params)]
+        L.siac_eval.restype = ctypes.c_int
+        L.siac_eval.argtypes = [vp, D, I64, D]
+        L.siac_eval_async.restype = ctypes.c_int
+        L.siac_eval_async.argtypes = [vp, vp, I64, vp, vp]
+        L.siac_set_counting.restype = ctypes.c_int
+        L.siac_set_counting.argtypes = [vp, I32]
+        L.siac_stats.restype = ctypes.c_int
+        L.siac_stats.argtypes = [vp, ctypes.POINTER(_Counters)]
+        L.siac_set_timing.restype = ctypes.c_int
+        L.siac_set_timing.argtypes = [vp, I32]
+        L.siac_timing.restype = ctypes.c_int
+        L.siac_timing.argtypes = [vp, D, ctypes.POINTER(I64)]
+        L.siac_probe_fp64.restype = ctypes.c_int
+        L.siac_probe_fp64.argtypes = [I32, D]
+        L.siac_info.restype = ctypes.c_int
+        L.siac_info.argtypes = [vp, ctypes.POINTER(I64), ctypes.POINTER(I32), ctypes.POINTER(I32),
+                                D, D]
+        L.siac_host_tables.restype = ctypes.c_int
+        L.siac_host_tables.argtypes = [I32, D, D]
+        L.siac_debug_records.restype = ctypes.c_int
+        L.siac_debug_records.argtypes = [vp, I64, D, ctypes.POINTER(I32)]
+        L.siac_destroy.restype = None
+        L.siac_destroy.argtypes = [vp]
+        L.siac_last_error.restype = ctypes.c_char_p
+        L.siac_last_error.argtypes = [vp]
+        L.siac_version.restype = ctypes.c_char_p
+        L.siac_version.argtypes = []
+        _lib = L
+    return _lib
+
+
+EXPORTED = ["siac_create", "siac_eval", "siac_eval_async", "siac_set_counting", "siac_stats",
+            "siac_set_timing", "siac_timing", "siac_probe_fp64",
+            "siac_info", "siac_host_tables", "siac_debug_records",
+            "siac_destroy", "siac_last_error", "siac_version"]
+
+
+def _dp(a):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
+
+
+def _check(rc, ctx_ptr=None):
+    if rc != 0:
+        msg = lib().siac_last_error(ctx_ptr).decode()
+        raise SiacError(f"siac error {rc}: {msg}")
+
+
+class Context:
+    """A siac_ctx: device-resident mesh + spatial index."""
+
+    def __init__(self, V, T, C, k: int, h: float, periodic: int = 3, domain=(0.0, 0.0, 1.0, 1.0),
+                 device: int = 0, cell_factor: float = 0.0):
+        L = lib()
+        self._V = np.ascontiguousarray(V, dtype=np.float64)
+        self._T = np.ascontiguousarray(T, dtype=np.int32)
+        self._C = np.ascontiguousarray(C, dtype=np.float64)
+        p = _Params(int(k), float(h), int(periodic), (ctypes.c_double * 4)(*domain), int(device), float(cell_factor))
+        ptr = ctypes.c_void_p()
+        rc = L.siac_create(ctypes.byref(ptr), _dp(self._V), len(self._V),
+                           self._T.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)), len(self._T),
+                           _dp(self._C), ctypes.byref(p))
+        _check(rc, None)
+        self._ptr = ptr
+        self.k, self.h, self.periodic, self.domain, self.device = int(k), float(h), int(periodic), tuple(domain), device
+        del self._V, self._T, self._C     # siac_create deep-copied them
+
+    def eval(self, points) -> np.ndarray:
+        """siac_eval: host points (n,2) -> host values (n,), H2D/D2H inside."""
+        P = np.ascontiguousarray(points, dtype=np.float64).reshape(-1, 2)
+        out = np.empty(len(P), dtype=np.float64)
+        _check(lib().siac_eval(self._ptr, _dp(P), len(P), _dp(out)), self._ptr)
+        return out
+
+    def eval_into(self, points: np.ndarray, out: np.ndarray) -> None:
+        """siac_eval into caller-owned host arrays (e.g. pinned torch tensors' numpy views)."""
+        _check(lib().siac_eval(self._ptr, _dp(points), len(points), _dp(out)), self._ptr)
+
+    def eval_async(self, d_points, d_out, stream=None) -> None:
+        """siac_eval_async on device memory: d_points / d_out are CUDA tensors (float64) or raw
+        device pointers (ints); stream is a torch.cuda.Stream, a raw cudaStream_t int, or None
+        (the current torch stream when tensors are given)."""
+        n = None
+        if hasattr(d_points, "data_ptr"):
+            assert d_points.dtype.is_floating_point and d_points.element_size() == 8 and d_points.is_contiguous()
+            assert d_out.element_size() == 8 and d_out.is_contiguous()
+            n = d_points.numel() // 2
+            assert d_out.numel() >= n
+            pp, po = d_points.data_ptr(), d_out.data_ptr()
+            if stream is None:
+                import torch
+                stream = torch.cuda.current_stream(d_points.device)
+        else:
+            raise TypeError("pass CUDA tensors (use eval_ptr for raw pointers)")
+        sh = stream.cuda_stream if hasattr(stream, "cuda_stream") else (stream or 0)
+        _check(lib().siac_eval_async(self._ptr, ctypes.c_void_p(pp), n, ctypes.c_void_p(po), ctypes.c_void_p(sh)),
+               self._ptr)
+
+    def eval_ptr(self, d_points: int, n: int, d_out: int, stream: int = 0) -> None:
+        _check(lib().siac_eval_async(self._ptr, ctypes.c_void_p(d_points), int(n), ctypes.c_void_p(d_out),
+                                     ctypes.c_void_p(stream)), self._ptr)
+
+    def set_counting(self, on: bool = True) -> None:
+        _check(lib().siac_set_counting(self._ptr, 1 if on else 0), self._ptr)
+
+    def stats(self) -> dict:
+        c = _Counters()
+        _check(lib().siac_stats(self._ptr, ctypes.byref(c)), self._ptr)
+        return {f: getattr(c, f) for f, _ in _Counters._fields_}
+
+    def set_timing(self, on: bool = True) -> None:
+        _check(lib().siac_set_timing(self._ptr, 1 if on else 0), self._ptr)
+
+    def timing(self) -> tuple[float, int]:
+        """(sum of main-kernel ms, number of timed launches) since the last call."""
+        ms, n = ctypes.c_double(), ctypes.c_int64()
+        _check(lib().siac_timing(self._ptr, ctypes.byref(ms), ctypes.byref(n)), self._ptr)
+        return ms.value, n.value
+
+    def info(self) -> dict:
+        nt, gx, gy = ctypes.c_int64(), ctypes.c_int32(), ctypes.c_int32()
+        cw, ch = ctypes.c_double(), ctypes.c_double()
+        _check(lib().siac_info(self._ptr, ctypes.byref(nt), ctypes.byref(gx), ctypes.byref(gy),
+                               ctypes.byref(cw), ctypes.byref(ch)), self._ptr)
+        return dict(n_triangles=nt.value, grid_nx=gx.value, grid_ny=gy.value, cell_w=cw.value, cell_h=ch.value)
+
+    def debug_records(self, n: int) -> np.ndarray:
+        rd = ctypes.c_int32()
+        _check(lib().siac_debug_records(self._ptr, 0, None, ctypes.byref(rd)), self._ptr)
+        out = np.empty((n, rd.value))
+        _check(lib().siac_debug_records(self._ptr, n, _dp(out), ctypes.byref(rd)), self._ptr)
+        return out
+
+    def destroy(self) -> None:
+        if getattr(self, "_ptr", None):
+            lib().siac_destroy(self._ptr)
+            self._ptr = None
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.destroy()
+
+
+def create(V, T, C, k, h, periodic=3, domain=(0.0, 0.0, 1.0, 1.0), device=0, cell_factor=0.0) -> Context:
+    return Context(V, T, C, k, h, periodic, domain, device, cell_factor)
+
+
+def host_tables(k: int):
+    """(cell_table (3k+1, k+1), basis_matrix (nb, nb)) computed by the library's host code."""
+    nb = (k + 1) * (k + 2) // 2
+    t = np.empty((3 * k + 1, k + 1))
+    R = np.empty((nb, nb))
+    _check(lib().siac_host_tables(int(k), _dp(t), _dp(R)), None)
+    return t, R
+
+
+def probe_fp64(device: int = 0) -> float:
+    """Measured FP64 FMA throughput (TFLOP/s) of `device` (siac_probe_fp64)."""
+    t = ctypes.c_double()
+    _check(lib().siac_probe_fp64(int(device), ctypes.byref(t)), None)
+    return t.value
+
+
+def version() -> str:
+    return lib().siac_version().decode()

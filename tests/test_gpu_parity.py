@@ -1,0 +1,244 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, element by element.
+
+Tolerance (north_star: 1e-10 relative; rule from SURVEY §8(c.5)): PASS iff
+    max_i |g_i - o_i| <= 1e-10 * max_i |o_i|                      (normwise), and
+    |g_i - o_i| <= 1e-10 * |o_i|  for every i with |o_i| >= 1e-2 max|o|   (pointwise).
+Small configs are compared at every point; the large ones evaluate ALL points on the GPU
+in the bench's launch configuration and compare a deterministic sample the oracle can
+afford, plus points next to the domain boundary (periodic wrap) and mesh vertices.
+"""
+import math
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_0007k13_b200 import inputs
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-10
+
+
+def assert_parity(g, o, tol=TOL):
+    g, o = np.asarray(g), np.asarray(o)
+    assert g.shape == o.shape
+    assert np.all(np.isfinite(g))
+    scale = max(np.abs(o).max(), 1e-300)
+    err = np.abs(g - o)
+    assert err.max() <= tol * scale, f"normwise {err.max() / scale:.3e}"
+    big = np.abs(o) >= 1e-2 * scale
+    if big.any():
+        rel = err[big] / np.abs(o[big])
+        assert rel.max() <= tol, f"pointwise {rel.max():.3e}"
+
+
+@pytest.fixture(scope="module")
+def siac_mod():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_sc_0007k13_b200 import siac
+    siac.lib()
+    return siac
+
+
+_CFG = {}
+
+
+def cfg(c, field="sinsin"):
+    key = (c, field)
+    if key not in _CFG:
+        _CFG[key] = inputs.make_config(c, field_kind=field)
+    return _CFG[key]
+
+
+def gpu_eval(siac_mod, w, points=None, **kw):
+    ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h, periodic=w.periodic, domain=w.domain, **kw)
+    try:
+        return ctx.eval(w.points if points is None else points)
+    finally:
+        ctx.destroy()
+
+
+def sample_idx(n, m, seed):
+    rng = np.random.default_rng(seed)
+    return np.sort(rng.choice(n, size=min(n, m), replace=False))
+
+
+# ------------------------------------------------------------------ configs
+
+@pytest.mark.parametrize("field", ["sinsin", "random"])
+def test_cfg1_every_point(siac_mod, oracle_mod, field):
+    w = cfg(1, field)
+    assert_parity(gpu_eval(siac_mod, w), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points))
+
+
+@pytest.mark.parametrize("field", ["sinsin", "random"])
+def test_cfg2_every_point(siac_mod, oracle_mod, field):
+    w = cfg(2, field)
+    assert_parity(gpu_eval(siac_mod, w), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points))
+
+
+@pytest.mark.parametrize("c,m", [(3, 1200), (4, 400), (5, 1500)])
+def test_large_configs_sampled(siac_mod, oracle_mod, c, m):
+    """All points on the GPU (bench launch configuration), oracle on a deterministic sample
+    plus the points closest to the periodic boundary."""
+    w = cfg(c)
+    g = gpu_eval(siac_mod, w)
+    idx = sample_idx(w.n_points, m, seed=c)
+    edge = np.minimum.reduce([w.points[:, 0], 1 - w.points[:, 0], w.points[:, 1], 1 - w.points[:, 1]])
+    idx = np.unique(np.concatenate([idx, np.argsort(edge)[:100]]))
+    o = oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points[idx])
+    assert_parity(g[idx], o)
+
+
+def test_cfg5_random_field_sampled(siac_mod, oracle_mod):
+    w = cfg(5, "random")
+    g = gpu_eval(siac_mod, w)
+    idx = sample_idx(w.n_points, 800, seed=55)
+    assert_parity(g[idx], oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points[idx]))
+
+
+# ------------------------------------------------------------------ invariants at full size
+
+@pytest.mark.parametrize("c", [1, 2, 3, 4, 5])
+def test_constant_field_every_point(siac_mod, c):
+    """u = 1 -> u* = 1 at every point of every config (P3), any size."""
+    w = cfg(c)
+    C = np.zeros_like(w.C)
+    C[:, 0] = math.sqrt(2.0)
+    ctx = siac_mod.create(w.V, w.T, C, w.k, w.h)
+    g = ctx.eval(w.points)
+    ctx.destroy()
+    assert np.abs(g - 1.0).max() < 1e-12
+
+
+def test_deterministic_bitwise(siac_mod):
+    w = cfg(3)
+    ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
+    a = ctx.eval(w.points)
+    b = ctx.eval(w.points)
+    ctx.destroy()
+    assert np.array_equal(a, b)
+
+
+def test_counters(siac_mod):
+    w = cfg(2)
+    ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
+    ctx.set_counting(True)
+    ctx.eval(w.points)
+    s = ctx.stats()
+    ctx.destroy()
+    assert s["n_points"] == w.n_points
+    assert s["candidates"] >= s["pairs"] > 0
+    assert s["subtris"] >= s["pieces"] >= s["pairs"] * 0.9
+
+
+# ------------------------------------------------------------------ edge cases
+
+def test_random_points_anywhere_wrap(siac_mod, oracle_mod):
+    """Points outside [0,1)^2 wrap (periodic), including exact corners and edges."""
+    w = cfg(2, "random")
+    P = np.random.default_rng(1).uniform(-1.5, 2.5, (3000, 2))
+    P[:6] = [[0, 0], [1, 1], [1, 0], [0.5, 1.0], [-1e-17, 0.3], [0.999999999999, 0.2]]
+    assert_parity(gpu_eval(siac_mod, w, P), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, P))
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 4])
+def test_structured_breaklines_on_mesh_lines(siac_mod, oracle_mod, k):
+    """h = mesh spacing: kernel breaklines coincide with mesh lines (odd k) or mid-lines
+    (even k); points at vertices, edge midpoints and cell centres; random field."""
+    N = 16
+    V, T = inputs.structured_mesh(N)
+    C = inputs.random_modes(len(T), k, seed=k)
+    h = 1.0 / N
+    g1 = np.arange(0, N + 1) / N
+    g2 = (np.arange(0, N) + 0.5) / N
+    X = np.concatenate([g1, g2])
+    P = np.array([[x, y] for x in X[::3] for y in X[::2]])
+    ctx = siac_mod.create(V, T, C, k, h)
+    g = ctx.eval(P)
+    ctx.destroy()
+    assert_parity(g, oracle_mod.oracle_eval(V, T, C, k, h, P))
+
+
+def test_stencil_equals_period(siac_mod, oracle_mod):
+    """W = (3k+1)h = period (k=1, N=4, h=1/4): every triangle meets the stencil through
+    several periodic images (SURVEY A4 case)."""
+    V, T = inputs.structured_mesh(4)
+    C = inputs.random_modes(len(T), 1, seed=2)
+    P = np.random.default_rng(3).uniform(0, 1, (200, 2))
+    ctx = siac_mod.create(V, T, C, 1, 0.25)
+    g = ctx.eval(P)
+    ctx.destroy()
+    assert_parity(g, oracle_mod.oracle_eval(V, T, C, 1, 0.25, P))
+
+
+def test_non_periodic_zero_extension(siac_mod, oracle_mod):
+    V, T = inputs.lattice_delaunay_mesh(3000, seed=9)
+    k = 2
+    C = inputs.random_modes(len(T), k, seed=4)
+    h = inputs.max_edge(V, T)
+    P = np.random.default_rng(5).uniform(-0.2, 1.2, (1500, 2))
+    for per in (0, 1, 2):
+        ctx = siac_mod.create(V, T, C, k, h, periodic=per)
+        g = ctx.eval(P)
+        ctx.destroy()
+        assert_parity(g, oracle_mod.oracle_eval(V, T, C, k, h, P, periodic=per))
+
+
+def test_graded_small_h_and_large_h(siac_mod, oracle_mod):
+    """h other than the max edge: smaller (triangles span many kernel cells) and larger."""
+    V, T = inputs.lattice_delaunay_mesh(2000, seed=12, graded=True)
+    C = inputs.random_modes(len(T), 2, seed=6)
+    P = inputs.eval_points(V, T, 2)[::17]
+    for h in (0.25 * inputs.max_edge(V, T), 0.12):
+        ctx = siac_mod.create(V, T, C, 2, h)
+        g = ctx.eval(P)
+        ctx.destroy()
+        assert_parity(g, oracle_mod.oracle_eval(V, T, C, 2, h, P))
+
+
+def test_single_triangle_and_empty(siac_mod, oracle_mod):
+    V = np.array([[0.2, 0.3], [0.45, 0.31], [0.3, 0.5]])
+    T = np.array([[0, 1, 2]], dtype=np.int32)
+    C = inputs.random_modes(1, 3, seed=1)
+    P = np.random.default_rng(2).uniform(0, 1, (257, 2))
+    ctx = siac_mod.create(V, T, C, 3, 0.05, periodic=0)
+    assert ctx.eval(np.zeros((0, 2))).shape == (0,)
+    g = ctx.eval(P)
+    ctx.destroy()
+    assert_parity(g, oracle_mod.oracle_eval(V, T, C, 3, 0.05, P, periodic=0))
+    ctx0 = siac_mod.create(np.zeros((0, 2)), np.zeros((0, 3), np.int32), np.zeros((0, 3)), 1, 0.1)
+    assert np.all(ctx0.eval(P) == 0.0)
+    ctx0.destroy()
+
+
+@pytest.mark.parametrize("n", [1, 31, 32, 33, 1000, 4097])
+def test_ragged_point_counts(siac_mod, oracle_mod, n):
+    w = cfg(2, "random")
+    P = w.points[sample_idx(w.n_points, n, seed=n)]
+    assert_parity(gpu_eval(siac_mod, w, P), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, P))
+
+
+def test_async_torch_stream(siac_mod, oracle_mod):
+    import torch
+    w = cfg(1, "random")
+    ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        P = torch.from_numpy(w.points).cuda()
+        out = torch.empty(w.n_points, dtype=torch.float64, device="cuda")
+        ctx.eval_async(P, out)
+    s.synchronize()
+    assert_parity(out.cpu().numpy(), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points))
+    ctx.destroy()
+
+
+def test_cell_factor_invariance(siac_mod):
+    """Results do not depend on the binning cell size (P10), bitwise up to summation order."""
+    w = cfg(2, "random")
+    outs = []
+    for cf in (0.3, 0.5, 1.0, 2.0):
+        outs.append(gpu_eval(siac_mod, w, cell_factor=cf))
+    for o in outs[1:]:
+        assert np.abs(o - outs[0]).max() <= 1e-12 * np.abs(outs[0]).max()
