@@ -111,6 +111,16 @@ siac_status siac_eval(siac_ctx *ctx, const double *points_xy, int64_t n_points, 
 siac_status siac_eval_async(siac_ctx *ctx, const double *d_points_xy, int64_t n_points,
                             double *d_values_out, void *cuda_stream);
 
+/* Evaluation schedule (same result up to summation order):
+ *   SIAC_SCHEDULE_TILE  (0, default) one warp per tile of 32 Morton-ordered points; candidate
+ *                       test, Sutherland-Hodgman clipping and quadrature decoupled through
+ *                       per-warp shared-memory stacks so the FP64 quadrature runs on full warps;
+ *   SIAC_SCHEDULE_POINT (1) one thread per point, clip and integrate inline (the paper's
+ *                       per-point evaluation, Alg. 2, mapped one thread per point). */
+#define SIAC_SCHEDULE_TILE 0
+#define SIAC_SCHEDULE_POINT 1
+siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule);
+
 /* Enable (1) / disable (0) geometry counting in later evaluations (adds atomics; off by default). */
 siac_status siac_set_counting(siac_ctx *ctx, int32_t enable);
 

@@ -22,6 +22,7 @@
 
 #include "../../include/siac.h"
 #include "siac_device.cuh"
+#include "siac_tile.cuh"
 #include "siac_math.h"
 
 #define SIAC_VERSION "siac-b200 0.1 (sm_100a, fp64)"
@@ -53,6 +54,7 @@ struct siac_ctx {
     int64_t cap_host = 0;
     double *d_hpts = nullptr, *d_hout = nullptr;
     // counters
+    int schedule = 0;            // 0 = warp-per-tile (default), 1 = thread-per-point
     bool counting = false;
     unsigned long long *d_cnt = nullptr;
     int64_t last_np = 0;
@@ -113,13 +115,19 @@ __global__ void k_prep(PrepArgs a) {
     const double det = a11 * a22 - a12 * a21;
     const double f = 3.0 * a.h / det;
     r[6] = f * a22; r[7] = -f * a12; r[8] = -f * a21; r[9] = f * a11;
+    const double vx[3] = {v0x, v1x, v2x}, vy[3] = {v0y, v1y, v2y};
+    for (int g = 0; g < 3; ++g) {
+        const double dx = vx[(g + 1) % 3] - vx[g], dy = vy[(g + 1) % 3] - vy[g];
+        r[10 + g] = dy / dx;         // +-inf for a vertical edge (never used for vertical lines)
+        r[13 + g] = dx / dy;
+    }
     const double *c = a.C + (int64_t)a.nb * t;
     for (int j = 0; j < a.nb; ++j) {
         double s = 0.0;
         for (int i = 0; i < a.nb; ++i) s = fma(c[i], a.R[i * a.nb + j], s);
-        r[10 + j] = s;
+        r[16 + j] = s;
     }
-    for (int j = 10 + a.nb; j < a.rs; ++j) r[j] = 0.0;
+    for (int j = 16 + a.nb; j < a.rs; ++j) r[j] = 0.0;
     const double bx0 = fmin(v0x, fmin(v1x, v2x)), bx1 = fmax(v0x, fmax(v1x, v2x));
     const double by0 = fmin(v0y, fmin(v1y, v2y)), by1 = fmax(v0y, fmax(v1y, v2y));
     a.bbox[t] = make_double4(bx0, by0, bx1, by1);
@@ -253,7 +261,7 @@ __global__ void __launch_bounds__(128) k_eval_v1(EvalArgs a) {
                     g.zv0x = zx[0]; g.zv0y = zy[0];
                     double d[NB];
 #pragma unroll
-                    for (int m = 0; m < NB; ++m) d[m] = rc[10 + m];
+                    for (int m = 0; m < NB; ++m) d[m] = rc[Rec<K>::OFF_D + m];
                     acc += pair_contrib<K, COUNT>(zx, zy, kc, d, g, cnt);
                 }
                 C = cend + 1;
@@ -277,11 +285,26 @@ __global__ void __launch_bounds__(128) k_eval_v1(EvalArgs a) {
 }
 
 template <int K>
-void launch_eval(const EvalArgs &a, bool count, cudaStream_t st) {
-    const int bs = 128;
-    const unsigned grid = (unsigned)((a.np + bs - 1) / bs);
-    if (count) k_eval_v1<K, true><<<grid, bs, 0, st>>>(a);
-    else k_eval_v1<K, false><<<grid, bs, 0, st>>>(a);
+void launch_eval(const EvalArgs &a, bool count, int schedule, cudaStream_t st) {
+    if (schedule == 1) {
+        const int bs = 128;
+        const unsigned grid = (unsigned)((a.np + bs - 1) / bs);
+        if (count) k_eval_v1<K, true><<<grid, bs, 0, st>>>(a);
+        else k_eval_v1<K, false><<<grid, bs, 0, st>>>(a);
+        return;
+    }
+    siactile::TileArgs t;
+    t.pts = a.pts; t.perm = a.perm; t.np = a.np; t.out = a.out; t.rec = a.rec; t.bbox = a.bbox;
+    t.cell_start = a.cell_start; t.kc = a.kc; t.x0 = a.x0; t.y0 = a.y0; t.Lx = a.Lx; t.Ly = a.Ly;
+    t.inv_h = a.inv_h; t.hw = a.hw; t.cw = a.cw; t.chh = a.chh; t.ex = a.ex; t.ey = a.ey;
+    t.ncx = a.ncx; t.ncy = a.ncy; t.periodic = a.periodic; t.cnt = a.cnt;
+    const int64_t ntiles = (a.np + 31) / 32;
+    const unsigned grid = (unsigned)((ntiles + siactile::WARPS - 1) / siactile::WARPS);
+    const size_t smem = sizeof(siactile::WarpSmem) * siactile::WARPS;
+    if (count) CK(cudaFuncSetAttribute(siactile::k_eval_tile<K, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    else CK(cudaFuncSetAttribute(siactile::k_eval_tile<K, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    if (count) siactile::k_eval_tile<K, true><<<grid, siactile::WARPS * 32, smem, st>>>(t);
+    else siactile::k_eval_tile<K, false><<<grid, siactile::WARPS * 32, smem, st>>>(t);
 }
 
 inline unsigned nblk(int64_t n, int bs) { return (unsigned)((n + bs - 1) / bs); }
@@ -345,10 +368,10 @@ void eval_device(siac_ctx *c, const double *d_pts, int64_t np, double *d_out, cu
         ++c->ev_used;
     }
     switch (c->k) {
-        case 1: launch_eval<1>(a, c->counting, st); break;
-        case 2: launch_eval<2>(a, c->counting, st); break;
-        case 3: launch_eval<3>(a, c->counting, st); break;
-        case 4: launch_eval<4>(a, c->counting, st); break;
+        case 1: launch_eval<1>(a, c->counting, c->schedule, st); break;
+        case 2: launch_eval<2>(a, c->counting, c->schedule, st); break;
+        case 3: launch_eval<3>(a, c->counting, c->schedule, st); break;
+        case 4: launch_eval<4>(a, c->counting, c->schedule, st); break;
         default: throw Fail{SIAC_EINTERNAL, "bad k"};
     }
     CK(cudaGetLastError());
@@ -488,7 +511,7 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
             CK(cudaMemset(c->d_cell_start, 0, sizeof(int) * (ncell + 1)));
             return;
         }
-        const int rs = (10 + nb + 1) & ~1;
+        const int rs = (16 + nb + 1) & ~1;
         double *dV = nullptr, *dC = nullptr, *dR = nullptr, *rec_u = nullptr;
         int *dT = nullptr;
         double4 *bb_u = nullptr;
@@ -601,6 +624,13 @@ siac_status siac_stats(siac_ctx *ctx, siac_counters *out) {
     });
 }
 
+siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule) {
+    if (!ctx) { g_err = "NULL context"; return SIAC_EINVAL; }
+    if (schedule < 0 || schedule > 1) { ctx->err = "unknown schedule"; return SIAC_EINVAL; }
+    ctx->schedule = schedule;
+    return SIAC_OK;
+}
+
 siac_status siac_set_timing(siac_ctx *ctx, int32_t enable) {
     if (!ctx) { g_err = "NULL context"; return SIAC_EINVAL; }
     ctx->timing = enable != 0;
@@ -683,7 +713,7 @@ siac_status siac_debug_records(siac_ctx *ctx, int64_t n, double *out, int32_t *r
     if (!ctx) { g_err = "NULL context"; return SIAC_EINVAL; }
     return run_guarded(&ctx->err, [&]() {
         const int nb = (ctx->k + 1) * (ctx->k + 2) / 2;
-        const int rs = (10 + nb + 1) & ~1;
+        const int rs = (16 + nb + 1) & ~1;
         if (rd) *rd = rs;
         need(n >= 0 && n <= ctx->nt, "n out of range");
         if (n > 0 && out) {

@@ -43,14 +43,17 @@ template <int K> __device__ __forceinline__ double qw(int q) {
 
 // ------------------------------------------------------------------ record layout
 // Triangle record (doubles), sorted by anchor cell:
-//   [0..5]  v0x v0y v1x v1y v2x v2y         physical vertices (unshifted)
-//   [6..9]  M00 M01 M10 M11                  M = 3 h A^{-1}, A = [v1-v0 | v2-v0]:
+//   [0..5]   v0x v0y v1x v1y v2x v2y        physical vertices (unshifted)
+//   [6..9]   M00 M01 M10 M11                 M = 3 h A^{-1}, A = [v1-v0 | v2-v0]:
 //                                            (rho, sigma) = M (z - z_v0) - (1, 1)
-//   [10..]  d_ab                             u_T in centred coords rho = 3r-1, sigma = 3s-1,
+//   [10..12] dy/dx of edges 0, 1, 2          edge g runs from vertex g to vertex (g+1)%3
+//   [13..15] dx/dy of edges 0, 1, 2          (slopes are scale-invariant: same in the z-frame)
+//   [16..]   d_ab                            u_T in centred coords rho = 3r-1, sigma = 3s-1,
 //                                            Horner order (a = k..0, b = 0..k-a)
 template <int K> struct Rec {
     static constexpr int NB = (K + 1) * (K + 2) / 2;
-    static constexpr int RAW = 10 + NB;
+    static constexpr int OFF_D = 16;
+    static constexpr int RAW = OFF_D + NB;
     static constexpr int RS = (RAW + 1) & ~1;        // padded to 16 B
 };
 
@@ -124,19 +127,25 @@ constexpr int PCAP = 10;   // a triangle ∩ 4 half-planes has <= 7 vertices; ma
 // coord <= X (L) and coord >= X (R).  Each output is exactly Alg. 1's output for that clip
 // edge (vertices on the line belong to both; an intersection is added only where an edge
 // crosses the line strictly, so no duplicate vertices).  The crossing point is computed
-// from the same ordered edge for both outputs, so neighbouring pieces share it bit-exactly.
+// once from the ordered edge and given to both outputs, so neighbouring pieces share it
+// bit-exactly.  Two comparisons per vertex.
 template <int AX>
 __device__ __forceinline__ void split_poly(const double *px, const double *py, int n, double X,
                                            double *lx, double *ly, int &nl, double *rx, double *ry, int &nr) {
     nl = 0;
     nr = 0;
+    const double c0 = AX ? py[0] : px[0];
+    const bool le0 = c0 <= X, ge0 = c0 >= X;
+    bool le_e = le0, ge_e = ge0;
+    double ce = c0;
     for (int e = 0; e < n; ++e) {
         const int f = (e + 1 == n) ? 0 : e + 1;
-        const double ce = AX ? py[e] : px[e];
         const double cf = AX ? py[f] : px[f];
-        if (ce <= X && nl < PCAP) { lx[nl] = px[e]; ly[nl] = py[e]; ++nl; }
-        if (ce >= X && nr < PCAP) { rx[nr] = px[e]; ry[nr] = py[e]; ++nr; }
-        if ((ce < X && cf > X) || (ce > X && cf < X)) {
+        const bool le_f = (f == 0) ? le0 : (cf <= X);
+        const bool ge_f = (f == 0) ? ge0 : (cf >= X);
+        if (le_e && nl < PCAP) { lx[nl] = px[e]; ly[nl] = py[e]; ++nl; }
+        if (ge_e && nr < PCAP) { rx[nr] = px[e]; ry[nr] = py[e]; ++nr; }
+        if ((!ge_e && !le_f) || (!le_e && !ge_f)) {
             const double t = (X - ce) / (cf - ce);
             double ix, iy;
             if (AX == 0) { ix = X; iy = fma(t, py[f] - py[e], py[e]); }
@@ -144,6 +153,9 @@ __device__ __forceinline__ void split_poly(const double *px, const double *py, i
             if (nl < PCAP) { lx[nl] = ix; ly[nl] = iy; ++nl; }
             if (nr < PCAP) { rx[nr] = ix; ry[nr] = iy; ++nr; }
         }
+        le_e = le_f;
+        ge_e = ge_f;
+        ce = cf;
     }
 }
 
@@ -155,79 +167,79 @@ __device__ __forceinline__ int clampi(double v, int lo, int hi) {
 
 struct Counts { unsigned long long pairs, pieces, subtris; };
 
-// Contribution of one (point, triangle image) pair: clip the z-frame triangle against the
-// kernel cells it overlaps, fan-triangulate, integrate.  kc: (3K+1) x (K+1) cell table.
-template <int K, bool COUNT>
-__device__ double pair_contrib(const double *zx, const double *zy, const double *kc, const double *d,
-                               const PairGeom &g, Counts &cnt) {
+// Every non-empty piece (T ∩ kernel cell (i, j)) of the z-frame triangle (zx, zy), in column-
+// major cell order, passed to emit(px, py, n, i, j).  Columns are peeled off the remainder
+// polygon by vertical splits, rows off each column by horizontal splits (each split is one
+// Sutherland-Hodgman pass producing both sides); the parts outside the stencil
+// [T0, T0 + 3K+1]^2 are dropped.
+template <int K, class EMIT>
+__device__ __forceinline__ void gen_pieces(const double *zx, const double *zy, EMIT &emit) {
     constexpr int NC = 3 * K + 1;
     constexpr double T0 = -0.5 * (3 * K + 1);
     const double xmin = fmin(zx[0], fmin(zx[1], zx[2])), xmax = fmax(zx[0], fmax(zx[1], zx[2]));
     const int ilo = clampi(xmin - T0, 0, NC - 1), ihi = clampi(xmax - T0, 0, NC - 1);
-    double ax[PCAP], ay[PCAP];
+    double b0x[PCAP], b0y[PCAP], b1x[PCAP], b1y[PCAP], b2x[PCAP], b2y[PCAP], b3x[PCAP], b3y[PCAP];
+    double b4x[PCAP], b4y[PCAP];
+    double *ax = b0x, *ay = b0y, *fx = b1x, *fy = b1y;      // x-remainder and its spare buffer
     int na = 3;
     for (int v = 0; v < 3; ++v) { ax[v] = zx[v]; ay[v] = zy[v]; }
-    double tx_[PCAP], ty_[PCAP];
-    int nt_;
     if (xmin < T0) {           // drop the part left of the stencil
-        double lx[PCAP], ly[PCAP];
         int nl;
-        split_poly<0>(ax, ay, na, T0, lx, ly, nl, tx_, ty_, nt_);
-        for (int v = 0; v < nt_; ++v) { ax[v] = tx_[v]; ay[v] = ty_[v]; }
-        na = nt_;
+        split_poly<0>(ax, ay, na, T0, b4x, b4y, nl, fx, fy, na);
+        double *tx = ax, *ty = ay; ax = fx; ay = fy; fx = tx; fy = ty;
     }
-    double total = 0.0;
     for (int i = ilo; i <= ihi && na >= 3; ++i) {
         const double X1 = T0 + i + 1;
-        double cx_[PCAP], cy_[PCAP];
+        double *cx = b2x, *cy = b2y;       // column piece
         int nc;
         if (i < ihi || xmax > X1) {
-            split_poly<0>(ax, ay, na, X1, cx_, cy_, nc, tx_, ty_, nt_);
-            for (int v = 0; v < nt_; ++v) { ax[v] = tx_[v]; ay[v] = ty_[v]; }
-            na = nt_;
+            split_poly<0>(ax, ay, na, X1, cx, cy, nc, fx, fy, na);
+            double *tx = ax, *ty = ay; ax = fx; ay = fy; fx = tx; fy = ty;
         } else {
-            for (int v = 0; v < na; ++v) { cx_[v] = ax[v]; cy_[v] = ay[v]; }
-            nc = na;
-            na = 0;
+            cx = ax; cy = ay; nc = na; na = 0;
         }
         if (nc < 3) continue;
-        double ymin = cy_[0], ymax = cy_[0];
-        for (int v = 1; v < nc; ++v) { ymin = fmin(ymin, cy_[v]); ymax = fmax(ymax, cy_[v]); }
+        double ymin = cy[0], ymax = cy[0];
+        for (int v = 1; v < nc; ++v) { ymin = fmin(ymin, cy[v]); ymax = fmax(ymax, cy[v]); }
         const int jlo = clampi(ymin - T0, 0, NC - 1), jhi = clampi(ymax - T0, 0, NC - 1);
+        double *gx = (cx == b2x) ? b3x : b2x, *gy = (cx == b2x) ? b3y : b2y;   // spare for the y-remainder
         if (ymin < T0) {       // drop the part below the stencil
-            double lx[PCAP], ly[PCAP];
             int nl;
-            split_poly<1>(cx_, cy_, nc, T0, lx, ly, nl, tx_, ty_, nt_);
-            for (int v = 0; v < nt_; ++v) { cx_[v] = tx_[v]; cy_[v] = ty_[v]; }
-            nc = nt_;
+            split_poly<1>(cx, cy, nc, T0, b4x, b4y, nl, gx, gy, nc);
+            double *tx = cx, *ty = cy; cx = gx; cy = gy; gx = tx; gy = ty;
         }
-        double kx[K + 1];
-#pragma unroll
-        for (int m = 0; m <= K; ++m) kx[m] = kc[i * (K + 1) + m];
-        const double ccx = T0 + i + 0.5;
         for (int j = jlo; j <= jhi && nc >= 3; ++j) {
             const double Y1 = T0 + j + 1;
-            double qx_[PCAP], qy_[PCAP];
-            int nq;
             if (j < jhi || ymax > Y1) {
-                split_poly<1>(cx_, cy_, nc, Y1, qx_, qy_, nq, tx_, ty_, nt_);
-                for (int v = 0; v < nt_; ++v) { cx_[v] = tx_[v]; cy_[v] = ty_[v]; }
-                nc = nt_;
+                int nq;
+                split_poly<1>(cx, cy, nc, Y1, b4x, b4y, nq, gx, gy, nc);
+                double *tx = cx, *ty = cy; cx = gx; cy = gy; gx = tx; gy = ty;
+                if (nq >= 3) emit(b4x, b4y, nq, i, j);
             } else {
-                for (int v = 0; v < nc; ++v) { qx_[v] = cx_[v]; qy_[v] = cy_[v]; }
-                nq = nc;
+                if (nc >= 3) emit(cx, cy, nc, i, j);
                 nc = 0;
             }
-            if (nq < 3) continue;
-            double ky[K + 1];
-#pragma unroll
-            for (int m = 0; m <= K; ++m) ky[m] = kc[j * (K + 1) + m];
-            const double ccy = T0 + j + 0.5;
-            if (COUNT) { cnt.pieces++; cnt.subtris += nq - 2; }
-            for (int m = 1; m + 1 < nq; ++m)
-                total += integrate_subtri<K>(qx_[0], qy_[0], qx_[m], qy_[m], qx_[m + 1], qy_[m + 1], kx, ky, ccx, ccy, d, g);
         }
     }
+}
+
+// Contribution of one (point, triangle image) pair, integrated inline (thread-per-point
+// schedule).  kc: (3K+1) x (K+1) cell table.
+template <int K, bool COUNT>
+__device__ double pair_contrib(const double *zx, const double *zy, const double *kc, const double *d,
+                               const PairGeom &g, Counts &cnt) {
+    constexpr double T0 = -0.5 * (3 * K + 1);
+    double total = 0.0;
+    auto emit = [&](const double *qx, const double *qy, int nq, int i, int j) {
+        double kx[K + 1], ky[K + 1];
+#pragma unroll
+        for (int m = 0; m <= K; ++m) { kx[m] = kc[i * (K + 1) + m]; ky[m] = kc[j * (K + 1) + m]; }
+        if (COUNT) { cnt.pieces++; cnt.subtris += nq - 2; }
+        for (int m = 1; m + 1 < nq; ++m)
+            total += integrate_subtri<K>(qx[0], qy[0], qx[m], qy[m], qx[m + 1], qy[m + 1], kx, ky, T0 + i + 0.5,
+                                         T0 + j + 0.5, d, g);
+    };
+    gen_pieces<K>(zx, zy, emit);
     return total;
 }
 

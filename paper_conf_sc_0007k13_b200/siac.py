@@ -19,8 +19,8 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libsiac_b200.so")
-SOURCES = [os.path.join(_HERE, "csrc", f) for f in ("siac.cu", "siac_device.cuh", "siac_math.cpp", "siac_math.h",
-                                                    "siac_quadrature.h")]
+SOURCES = [os.path.join(_HERE, "csrc", f) for f in ("siac.cu", "siac_device.cuh", "siac_tile.cuh", "siac_clipfast.cuh", "siac_math.cpp",
+                                                    "siac_math.h", "siac_quadrature.h")]
 SOURCES.append(os.path.join(os.path.dirname(_HERE), "include", "siac.h"))
 
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
@@ -82,6 +82,8 @@ def lib():
         L.siac_set_counting.argtypes = [vp, I32]
         L.siac_stats.restype = ctypes.c_int
         L.siac_stats.argtypes = [vp, ctypes.POINTER(_Counters)]
+        L.siac_set_schedule.restype = ctypes.c_int
+        L.siac_set_schedule.argtypes = [vp, I32]
         L.siac_set_timing.restype = ctypes.c_int
         L.siac_set_timing.argtypes = [vp, I32]
         L.siac_timing.restype = ctypes.c_int
@@ -106,7 +108,7 @@ def lib():
 
 
 EXPORTED = ["siac_create", "siac_eval", "siac_eval_async", "siac_set_counting", "siac_stats",
-            "siac_set_timing", "siac_timing", "siac_probe_fp64",
+            "siac_set_schedule", "siac_set_timing", "siac_timing", "siac_probe_fp64",
             "siac_info", "siac_host_tables", "siac_debug_records",
             "siac_destroy", "siac_last_error", "siac_version"]
 
@@ -182,6 +184,10 @@ class Context:
         c = _Counters()
         _check(lib().siac_stats(self._ptr, ctypes.byref(c)), self._ptr)
         return {f: getattr(c, f) for f, _ in _Counters._fields_}
+
+    def set_schedule(self, schedule: int) -> None:
+        """0 = warp-per-tile (default), 1 = thread-per-point."""
+        _check(lib().siac_set_schedule(self._ptr, int(schedule)), self._ptr)
 
     def set_timing(self, on: bool = True) -> None:
         _check(lib().siac_set_timing(self._ptr, 1 if on else 0), self._ptr)

@@ -51,8 +51,9 @@ def cfg(c, field="sinsin"):
     return _CFG[key]
 
 
-def gpu_eval(siac_mod, w, points=None, **kw):
+def gpu_eval(siac_mod, w, points=None, schedule=0, **kw):
     ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h, periodic=w.periodic, domain=w.domain, **kw)
+    ctx.set_schedule(schedule)
     try:
         return ctx.eval(w.points if points is None else points)
     finally:
@@ -76,6 +77,14 @@ def test_cfg1_every_point(siac_mod, oracle_mod, field):
 def test_cfg2_every_point(siac_mod, oracle_mod, field):
     w = cfg(2, field)
     assert_parity(gpu_eval(siac_mod, w), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points))
+
+
+@pytest.mark.parametrize("c", [1, 2])
+def test_point_schedule_matches_oracle(siac_mod, oracle_mod, c):
+    """The thread-per-point schedule (SIAC_SCHEDULE_POINT) computes the same values."""
+    w = cfg(c, "random")
+    o = oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points)
+    assert_parity(gpu_eval(siac_mod, w, schedule=1), o)
 
 
 @pytest.mark.parametrize("c,m", [(3, 1200), (4, 400), (5, 1500)])
@@ -121,16 +130,24 @@ def test_deterministic_bitwise(siac_mod):
     assert np.array_equal(a, b)
 
 
-def test_counters(siac_mod):
+def test_counters_agree_between_schedules(siac_mod):
+    """Both schedules clip the same pieces: pairs, pieces and sub-triangles agree."""
     w = cfg(2)
     ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
     ctx.set_counting(True)
-    ctx.eval(w.points)
-    s = ctx.stats()
+    got = []
+    for sch in (0, 1):
+        ctx.set_schedule(sch)
+        ctx.eval(w.points)
+        got.append(ctx.stats())
     ctx.destroy()
+    s = got[0]
     assert s["n_points"] == w.n_points
     assert s["candidates"] >= s["pairs"] > 0
     assert s["subtris"] >= s["pieces"] >= s["pairs"] * 0.9
+    assert got[0]["pairs"] == got[1]["pairs"]
+    assert abs(got[0]["pieces"] - got[1]["pieces"]) <= 1e-4 * got[1]["pieces"]
+    assert abs(got[0]["subtris"] - got[1]["subtris"]) <= 1e-4 * got[1]["subtris"]
 
 
 # ------------------------------------------------------------------ edge cases
