@@ -279,7 +279,7 @@ def run_siac(args):
                              "algorithmic_flops_per_step": flops_step},
                 "e2e": {"value": e2e_val, "unit": "points/s", "h2d_bytes_per_step": int(w.n_points * 16),
                         "d2h_bytes_per_step": int(w.n_points * 8)},
-                "schedule": ["tile", "point"][args.schedule],
+                "schedule": ["default(tile)", "point", "tile", "ws"][args.schedule],
                 "gpu_launches": 2 * args.steps,
                 "gpu_launches_note": "per step: k_point_keys + k_eval (ours) + CUB radix-sort kernels (library)",
                 "clocks": clk}
@@ -303,7 +303,8 @@ def main():
     ap.add_argument("--impl", default="siac", choices=["siac", "reference"])
     ap.add_argument("--ref-points", type=int, default=4000, help="oracle sample size (points)")
     ap.add_argument("--e2e-steps", type=int, default=3)
-    ap.add_argument("--schedule", type=int, default=0, help="0 = warp-per-tile (default), 1 = thread-per-point")
+    ap.add_argument("--schedule", type=int, default=0,
+                    help="0 = default, 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:

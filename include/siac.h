@@ -112,13 +112,18 @@ siac_status siac_eval_async(siac_ctx *ctx, const double *d_points_xy, int64_t n_
                             double *d_values_out, void *cuda_stream);
 
 /* Evaluation schedule (same result up to summation order):
- *   SIAC_SCHEDULE_TILE  (0, default) one warp per tile of 32 Morton-ordered points; candidate
- *                       test, Sutherland-Hodgman clipping and quadrature decoupled through
- *                       per-warp shared-memory stacks so the FP64 quadrature runs on full warps;
- *   SIAC_SCHEDULE_POINT (1) one thread per point, clip and integrate inline (the paper's
- *                       per-point evaluation, Alg. 2, mapped one thread per point). */
-#define SIAC_SCHEDULE_TILE 0
+ *   SIAC_SCHEDULE_DEFAULT (0) the fastest measured schedule (currently SIAC_SCHEDULE_TILE);
+ *   SIAC_SCHEDULE_POINT   (1) one thread per point, clip and integrate inline (the paper's
+ *                         per-point evaluation, Alg. 2, one thread per point);
+ *   SIAC_SCHEDULE_TILE    (2) one warp per tile of 32 Morton-ordered points: ballot-compacted
+ *                         candidate tests, register-only Sutherland-Hodgman splits, sub-triangles
+ *                         staged in shared memory and integrated 32 at a time by the full warp;
+ *   SIAC_SCHEDULE_WS      (3) persistent warp-specialized variant of TILE: producer warps clip,
+ *                         paired consumer warps integrate double-buffered batches (mbarriers). */
+#define SIAC_SCHEDULE_DEFAULT 0
 #define SIAC_SCHEDULE_POINT 1
+#define SIAC_SCHEDULE_TILE 2
+#define SIAC_SCHEDULE_WS 3
 siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule);
 
 /* Enable (1) / disable (0) geometry counting in later evaluations (adds atomics; off by default). */

@@ -23,6 +23,7 @@
 #include "../../include/siac.h"
 #include "siac_device.cuh"
 #include "siac_tile.cuh"
+#include "siac_ws.cuh"
 #include "siac_math.h"
 
 #define SIAC_VERSION "siac-b200 0.1 (sm_100a, fp64)"
@@ -54,7 +55,9 @@ struct siac_ctx {
     int64_t cap_host = 0;
     double *d_hpts = nullptr, *d_hout = nullptr;
     // counters
-    int schedule = 0;            // 0 = warp-per-tile (default), 1 = thread-per-point
+    int schedule = 0;            // 0 = default (= 2), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized
+    int *d_tile_counter = nullptr;
+    int num_sms = 148;
     bool counting = false;
     unsigned long long *d_cnt = nullptr;
     int64_t last_np = 0;
@@ -285,7 +288,27 @@ __global__ void __launch_bounds__(128) k_eval_v1(EvalArgs a) {
 }
 
 template <int K>
-void launch_eval(const EvalArgs &a, bool count, int schedule, cudaStream_t st) {
+void launch_eval(const EvalArgs &a, bool count, int schedule, int *tile_counter, int num_sms, cudaStream_t st) {
+    if (schedule == 0) schedule = 2;     // the default schedule
+    if (schedule == 3) {
+        siacws::WsArgs w;
+        w.pts = a.pts; w.perm = a.perm; w.np = a.np; w.out = a.out; w.rec = a.rec; w.bbox = a.bbox;
+        w.cell_start = a.cell_start; w.kc = a.kc; w.x0 = a.x0; w.y0 = a.y0; w.Lx = a.Lx; w.Ly = a.Ly;
+        w.inv_h = a.inv_h; w.hw = a.hw; w.cw = a.cw; w.chh = a.chh; w.ex = a.ex; w.ey = a.ey;
+        w.ncx = a.ncx; w.ncy = a.ncy; w.periodic = a.periodic; w.cnt = a.cnt; w.tile_counter = tile_counter;
+        CK(cudaMemsetAsync(tile_counter, 0, sizeof(int), st));
+        const size_t smem = sizeof(siacws::Smem<K>);
+        const int64_t ntiles = (a.np + 31) / 32;
+        const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(num_sms, ntiles));
+        if (count) {
+            CK(cudaFuncSetAttribute(siacws::k_eval_ws<K, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            siacws::k_eval_ws<K, true><<<grid, siacws::NWARPS * 32, smem, st>>>(w);
+        } else {
+            CK(cudaFuncSetAttribute(siacws::k_eval_ws<K, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            siacws::k_eval_ws<K, false><<<grid, siacws::NWARPS * 32, smem, st>>>(w);
+        }
+        return;
+    }
     if (schedule == 1) {
         const int bs = 128;
         const unsigned grid = (unsigned)((a.np + bs - 1) / bs);
@@ -368,10 +391,10 @@ void eval_device(siac_ctx *c, const double *d_pts, int64_t np, double *d_out, cu
         ++c->ev_used;
     }
     switch (c->k) {
-        case 1: launch_eval<1>(a, c->counting, c->schedule, st); break;
-        case 2: launch_eval<2>(a, c->counting, c->schedule, st); break;
-        case 3: launch_eval<3>(a, c->counting, c->schedule, st); break;
-        case 4: launch_eval<4>(a, c->counting, c->schedule, st); break;
+        case 1: launch_eval<1>(a, c->counting, c->schedule, c->d_tile_counter, c->num_sms, st); break;
+        case 2: launch_eval<2>(a, c->counting, c->schedule, c->d_tile_counter, c->num_sms, st); break;
+        case 3: launch_eval<3>(a, c->counting, c->schedule, c->d_tile_counter, c->num_sms, st); break;
+        case 4: launch_eval<4>(a, c->counting, c->schedule, c->d_tile_counter, c->num_sms, st); break;
         default: throw Fail{SIAC_EINTERNAL, "bad k"};
     }
     CK(cudaGetLastError());
@@ -399,7 +422,7 @@ void free_ctx(siac_ctx *c) {
     cudaSetDevice(c->device);
     for (auto &e : c->ev) { cudaEventDestroy(e.first); cudaEventDestroy(e.second); }
     void *ptrs[] = {c->d_rec, c->d_bbox, c->d_cell_start, c->d_kc, c->d_keys[0], c->d_keys[1],
-                    c->d_idx[0], c->d_idx[1], c->d_cub, c->d_hpts, c->d_hout, c->d_cnt};
+                    c->d_idx[0], c->d_idx[1], c->d_cub, c->d_hpts, c->d_hout, c->d_cnt, c->d_tile_counter};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     delete c;
@@ -504,6 +527,8 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
         CK(cudaMalloc(&c->d_kc, sizeof(double) * kc.size()));
         CK(cudaMemcpy(c->d_kc, kc.data(), sizeof(double) * kc.size(), cudaMemcpyHostToDevice));
         CK(cudaMalloc(&c->d_cnt, 4 * sizeof(unsigned long long)));
+        CK(cudaMalloc(&c->d_tile_counter, sizeof(int)));
+        c->num_sms = prop.multiProcessorCount;
         CK(cudaMemset(c->d_cnt, 0, 4 * sizeof(unsigned long long)));
         const int64_t ncell = (int64_t)c->ncx * c->ncy;
         CK(cudaMalloc(&c->d_cell_start, sizeof(int) * (ncell + 1)));
@@ -626,7 +651,7 @@ siac_status siac_stats(siac_ctx *ctx, siac_counters *out) {
 
 siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule) {
     if (!ctx) { g_err = "NULL context"; return SIAC_EINVAL; }
-    if (schedule < 0 || schedule > 1) { ctx->err = "unknown schedule"; return SIAC_EINVAL; }
+    if (schedule < 0 || schedule > 3) { ctx->err = "unknown schedule"; return SIAC_EINVAL; }
     ctx->schedule = schedule;
     return SIAC_OK;
 }

@@ -119,6 +119,60 @@ __device__ __forceinline__ double integrate_subtri(double p0x, double p0y, doubl
     return area * acc;
 }
 
+// N independent sub-triangles integrated together: the quadrature loop runs over the rule
+// points outermost and the N sub-triangles innermost, so their FMA chains interleave
+// (instruction-level parallelism for a single warp feeding the FP64 pipe).
+#ifndef SIAC_QP_UNROLL
+#define SIAC_QP_UNROLL 64
+#endif
+constexpr int kQpUnroll = SIAC_QP_UNROLL;
+
+template <int K> struct SubTri {
+    double p0x, p0y, e1x, e1y, e2x, e2y;
+    double kx[K + 1], ky[K + 1];
+    double cx, cy;
+    double d[(K + 1) * (K + 2) / 2];
+    PairGeom g;
+};
+
+template <int K, int N>
+__device__ __forceinline__ void integrate_subtri_n(const SubTri<K> *t, double *out) {
+    double ax0[N], ay0[N], r0[N], rr[N], rs[N], s0[N], sr[N], ss[N], acc[N], area[N];
+#pragma unroll
+    for (int n = 0; n < N; ++n) {
+        const SubTri<K> &T = t[n];
+        area[n] = 0.5 * fabs(T.e1x * T.e2y - T.e1y * T.e2x);
+        ax0[n] = T.p0x - T.cx;
+        ay0[n] = T.p0y - T.cy;
+        const double dx0 = T.p0x - T.g.zv0x, dy0 = T.p0y - T.g.zv0y;
+        r0[n] = fma(T.g.M00, dx0, fma(T.g.M01, dy0, -1.0));
+        rr[n] = fma(T.g.M00, T.e1x, T.g.M01 * T.e1y);
+        rs[n] = fma(T.g.M00, T.e2x, T.g.M01 * T.e2y);
+        s0[n] = fma(T.g.M10, dx0, fma(T.g.M11, dy0, -1.0));
+        sr[n] = fma(T.g.M10, T.e1x, T.g.M11 * T.e1y);
+        ss[n] = fma(T.g.M10, T.e2x, T.g.M11 * T.e2y);
+        acc[n] = 0.0;
+    }
+    // rule points in a rolled loop (constant-bank loads): keeps the kernel small enough for
+    // the instruction cache, which a fully unrolled 19/33-point loop per sub-triangle is not
+#pragma unroll kQpUnroll
+    for (int q = 0; q < Rule<K>::NQ; ++q) {
+        const double r = qr<K>(q), s = qs<K>(q), w = qw<K>(q);
+#pragma unroll
+        for (int n = 0; n < N; ++n) {
+            const SubTri<K> &T = t[n];
+            const double tx = fma(T.e2x, s, fma(T.e1x, r, ax0[n]));
+            const double ty = fma(T.e2y, s, fma(T.e1y, r, ay0[n]));
+            const double rho = fma(rs[n], s, fma(rr[n], r, r0[n]));
+            const double sig = fma(ss[n], s, fma(sr[n], r, s0[n]));
+            const double kv = horner1<K>(T.kx, tx) * horner1<K>(T.ky, ty);
+            acc[n] = fma(w, kv * horner2<K>(T.d, rho, sig), acc[n]);
+        }
+    }
+#pragma unroll
+    for (int n = 0; n < N; ++n) out[n] = area[n] * acc[n];
+}
+
 // ------------------------------------------------------------------ Sutherland-Hodgman split
 
 constexpr int PCAP = 10;   // a triangle ∩ 4 half-planes has <= 7 vertices; margin for rounding

@@ -26,8 +26,17 @@ namespace siactile {
 
 using namespace siacdev;
 
-constexpr int WARPS = 4;        // warps per block
-constexpr int SLOTS = 8;        // sub-triangles a lane may stage per generation step
+#ifndef SIAC_TILE_WARPS
+#define SIAC_TILE_WARPS 4
+#endif
+#ifndef SIAC_TILE_SLOTS
+#define SIAC_TILE_SLOTS 8
+#endif
+#ifndef SIAC_TILE_MINB
+#define SIAC_TILE_MINB 3
+#endif
+constexpr int WARPS = SIAC_TILE_WARPS;   // warps per block
+constexpr int SLOTS = SIAC_TILE_SLOTS;   // sub-triangles a lane may stage per generation step
 constexpr int PSTACK = 64;      // pair stack: 31 left over + 32 new
 
 // Triangle record layout: siacdev::Rec (siac_device.cuh).
@@ -98,14 +107,14 @@ __device__ __forceinline__ void seg_add(WarpSmem &S, int key, double v, int lane
 template <int K>
 __device__ __forceinline__ void pair_data(const TileArgs &a, const WarpSmem &S, int tri, int pinfo, PairGeom &g,
                                           double *d) {
-    const double *rc = a.rec + (int64_t)Rec<K>::RS * tri;
+    const double *__restrict__ rc = a.rec + (int64_t)Rec<K>::RS * tri;
     const int slot = pinfo & 31, code = pinfo >> 5;
     const double psx = (double)(code % 3 - 1) * a.Lx, psy = (double)(code / 3 - 1) * a.Ly;
-    g.zv0x = ((rc[0] + psx) - S.px[slot]) * a.inv_h;
-    g.zv0y = ((rc[1] + psy) - S.py[slot]) * a.inv_h;
-    g.M00 = rc[6]; g.M01 = rc[7]; g.M10 = rc[8]; g.M11 = rc[9];
+    g.zv0x = ((__ldg(rc + 0) + psx) - S.px[slot]) * a.inv_h;
+    g.zv0y = ((__ldg(rc + 1) + psy) - S.py[slot]) * a.inv_h;
+    g.M00 = __ldg(rc + 6); g.M01 = __ldg(rc + 7); g.M10 = __ldg(rc + 8); g.M11 = __ldg(rc + 9);
 #pragma unroll
-    for (int m = 0; m < Rec<K>::NB; ++m) d[m] = rc[Rec<K>::OFF_D + m];
+    for (int m = 0; m < Rec<K>::NB; ++m) d[m] = __ldg(rc + Rec<K>::OFF_D + m);
 }
 
 // General splitter for pairs outside the fast path (h smaller than the triangles, or a
@@ -145,7 +154,7 @@ __device__ __noinline__ void gen_general(const TileArgs &a, WarpSmem &S, const d
 }
 
 template <int K, bool COUNT>
-__global__ void __launch_bounds__(WARPS * 32, 3) k_eval_tile(TileArgs a) {
+__global__ void __launch_bounds__(WARPS * 32, SIAC_TILE_MINB) k_eval_tile(TileArgs a) {
     constexpr int NC = 3 * K + 1;
     constexpr int NB = Rec<K>::NB;
     constexpr double T0 = -0.5 * (3 * K + 1);
@@ -263,16 +272,16 @@ __global__ void __launch_bounds__(WARPS * 32, 3) k_eval_tile(TileArgs a) {
             S.ginfo[lane] = pinfo;
             my_pinfo = pinfo & 31;
             const int slot = pinfo & 31, pcode = pinfo >> 5;
-            const double *rc = a.rec + (int64_t)Rec<K>::RS * tri;
+            const double *__restrict__ rc = a.rec + (int64_t)Rec<K>::RS * tri;
             const double psx = (double)(pcode % 3 - 1) * a.Lx, psy = (double)(pcode / 3 - 1) * a.Ly;
             const double px = S.px[slot], py = S.py[slot];
             siacfast::TriZ TZ;
 #pragma unroll
             for (int v = 0; v < 3; ++v) {
-                TZ.x[v] = ((rc[2 * v] + psx) - px) * a.inv_h;
-                TZ.y[v] = ((rc[2 * v + 1] + psy) - py) * a.inv_h;
-                TZ.syx[v] = rc[10 + v];
-                TZ.sxy[v] = rc[13 + v];
+                TZ.x[v] = ((__ldg(rc + 2 * v) + psx) - px) * a.inv_h;
+                TZ.y[v] = ((__ldg(rc + 2 * v + 1) + psy) - py) * a.inv_h;
+                TZ.syx[v] = __ldg(rc + 10 + v);
+                TZ.sxy[v] = __ldg(rc + 13 + v);
             }
             unsigned long long f_pieces = 0, f_sub = 0;
             auto emit_fast = [&](const siacfast::Poly &P, int i, int j) {

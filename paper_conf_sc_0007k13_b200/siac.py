@@ -19,7 +19,10 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libsiac_b200.so")
-SOURCES = [os.path.join(_HERE, "csrc", f) for f in ("siac.cu", "siac_device.cuh", "siac_tile.cuh", "siac_clipfast.cuh", "siac_math.cpp",
+# experiments only: SIAC_LIB_VARIANT=name loads libsiac_b200.<name>.so (built by tools/build_variant.py)
+if os.environ.get("SIAC_LIB_VARIANT"):
+    LIB_PATH = os.path.join(_HERE, f"libsiac_b200.{os.environ['SIAC_LIB_VARIANT']}.so")
+SOURCES = [os.path.join(_HERE, "csrc", f) for f in ("siac.cu", "siac_device.cuh", "siac_tile.cuh", "siac_ws.cuh", "siac_clipfast.cuh", "siac_math.cpp",
                                                     "siac_math.h", "siac_quadrature.h")]
 SOURCES.append(os.path.join(os.path.dirname(_HERE), "include", "siac.h"))
 
@@ -186,7 +189,7 @@ class Context:
         return {f: getattr(c, f) for f, _ in _Counters._fields_}
 
     def set_schedule(self, schedule: int) -> None:
-        """0 = warp-per-tile (default), 1 = thread-per-point."""
+        """0 = default (fastest), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized."""
         _check(lib().siac_set_schedule(self._ptr, int(schedule)), self._ptr)
 
     def set_timing(self, on: bool = True) -> None:

@@ -80,11 +80,12 @@ def test_cfg2_every_point(siac_mod, oracle_mod, field):
 
 
 @pytest.mark.parametrize("c", [1, 2])
-def test_point_schedule_matches_oracle(siac_mod, oracle_mod, c):
-    """The thread-per-point schedule (SIAC_SCHEDULE_POINT) computes the same values."""
+@pytest.mark.parametrize("schedule", [1, 2, 3])
+def test_every_schedule_matches_oracle(siac_mod, oracle_mod, c, schedule):
+    """Every schedule (point, tile, warp-specialized) computes the same values."""
     w = cfg(c, "random")
     o = oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points)
-    assert_parity(gpu_eval(siac_mod, w, schedule=1), o)
+    assert_parity(gpu_eval(siac_mod, w, schedule=schedule), o)
 
 
 @pytest.mark.parametrize("c,m", [(3, 1200), (4, 400), (5, 1500)])
@@ -136,7 +137,7 @@ def test_counters_agree_between_schedules(siac_mod):
     ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
     ctx.set_counting(True)
     got = []
-    for sch in (0, 1):
+    for sch in (0, 1, 3):
         ctx.set_schedule(sch)
         ctx.eval(w.points)
         got.append(ctx.stats())
@@ -145,9 +146,10 @@ def test_counters_agree_between_schedules(siac_mod):
     assert s["n_points"] == w.n_points
     assert s["candidates"] >= s["pairs"] > 0
     assert s["subtris"] >= s["pieces"] >= s["pairs"] * 0.9
-    assert got[0]["pairs"] == got[1]["pairs"]
-    assert abs(got[0]["pieces"] - got[1]["pieces"]) <= 1e-4 * got[1]["pieces"]
-    assert abs(got[0]["subtris"] - got[1]["subtris"]) <= 1e-4 * got[1]["subtris"]
+    for o in got[1:]:
+        assert got[0]["pairs"] == o["pairs"]
+        assert abs(got[0]["pieces"] - o["pieces"]) <= 1e-4 * o["pieces"]
+        assert abs(got[0]["subtris"] - o["subtris"]) <= 1e-4 * o["subtris"]
 
 
 # ------------------------------------------------------------------ edge cases
