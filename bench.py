@@ -107,8 +107,10 @@ def workload_desc(w, cfg):
 
 
 def cpu_baseline(w, sample_stride, nthreads=0):
-    """The oracle as it stands, on a deterministic stride sample of the workload's points."""
+    """The oracle as it stands, on a deterministic stride sample of the workload's points,
+    on all host cores (explicit: torchrun sets OMP_NUM_THREADS=1)."""
     import oracle
+    nthreads = nthreads or oracle.omp_threads()
     P = w.points[::sample_stride]
     t0 = time.perf_counter()
     oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P, nthreads=nthreads)
@@ -126,11 +128,11 @@ def run_reference(args):
     stride = max(1, w.n_points // args.ref_points)
     P = w.points[::stride]
     for _ in range(args.warmup):
-        oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P[:64])
+        oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P[:64], nthreads=oracle.omp_threads())
     times = []
     for _ in range(args.steps):
         t0 = time.perf_counter()
-        oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P)
+        oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P, nthreads=oracle.omp_threads())
         times.append(time.perf_counter() - t0)
     tot = sum(times)
     val = len(P) * args.steps / tot
@@ -155,23 +157,41 @@ def run_siac(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    dev = torch.device("cuda", local % max(ndev, 1))
     torch.cuda.set_device(dev)
+    backend = os.environ.get("SIAC_DIST_BACKEND", "nccl")     # gloo: functional runs with >1 rank per GPU
+    if world > 1:
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
+
+    def allreduce_max(vals):
+        if world == 1:
+            return vals
+        t = torch.tensor(vals, dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return t.tolist()
+
+    def allreduce_sum_int(vals):
+        if world == 1:
+            return vals
+        t = torch.tensor(vals, dtype=torch.int64, device=dev if backend == "nccl" else "cpu")
+        dist.all_reduce(t)
+        return [int(x) for x in t.tolist()]
 
     w = load_workload(args.config)
     k = w.k
     if world > 1:
         from paper_conf_sc_0007k13_b200 import dist as sdist
-        part = sdist.partition(w, world)
-        sub = sdist.local_problem(w, part, rank)
+        part = sdist.partition(w.points, world)
+        sub = sdist.local_problem(w.V, w.T, w.C, w.points, w.k, w.h, part, rank)
         V, T, C, P_local = sub["V"], sub["T"], sub["C"], sub["points"]
     else:
         part = None
         V, T, C, P_local = w.V, w.T, w.C, w.points
-    ctx = siac.create(V, T, C, k, w.h, periodic=3, device=local)
+    ctx = siac.create(V, T, C, k, w.h, periodic=3, device=dev.index)
     ctx.set_schedule(args.schedule)
     n_local = len(P_local)
     d_pts = torch.from_numpy(np.ascontiguousarray(P_local)).to(dev)
@@ -181,89 +201,94 @@ def run_siac(args):
     # geometry counts (untimed): the algorithmic flop count of the quadrature
     ctx.set_counting(True)
     ctx.eval_async(d_pts, d_out, stream)
-    stats = ctx.stats()
+    st = ctx.stats()
     ctx.set_counting(False)
-    subtris = stats["subtris"]
-    if world > 1:
-        t = torch.tensor([subtris, stats["pairs"], stats["pieces"], stats["candidates"]], dtype=torch.int64, device=dev)
-        dist.all_reduce(t)
-        subtris, pairs, pieces, cands = [int(x) for x in t.tolist()]
-    else:
-        pairs, pieces, cands = stats["pairs"], stats["pieces"], stats["candidates"]
+    cands, pairs, pieces, subtris = allreduce_sum_int([st["candidates"], st["pairs"], st["pieces"], st["subtris"]])
     flops_step = subtris * flops_per_subtri(k)           # whole job, per step
 
-    gathered = None
+    # per-step gather of the values (NCCL all_gather_into_tensor of padded slices)
     if world > 1:
         nmax = part["max_count"]
-        send = torch.zeros(nmax, dtype=torch.float64, device=dev)
-        gathered = torch.empty(world * nmax, dtype=torch.float64, device=dev)
+        gdev = dev if backend == "nccl" else torch.device("cpu")
+        send = torch.zeros(nmax, dtype=torch.float64, device=gdev)
+        gathered = torch.empty(world * nmax, dtype=torch.float64, device=gdev)
 
-    def step():
-        ctx.eval_async(d_pts, d_out, stream)
+    def gather(vals_dev):
         if world > 1:
-            send[:n_local].copy_(d_out[:n_local])
+            send[:n_local].copy_(vals_dev[:n_local])
             dist.all_gather_into_tensor(gathered, send)
 
+    # L2: flush between timed steps unless this rank's inputs alone exceed the 126 MB L2
+    rs = (16 + (k + 1) * (k + 2) // 2 + 1) & ~1
+    in_bytes = n_local * 16 + len(T) * rs * 8
+    flush = in_bytes < 2 * 126e6
+    scrub = torch.empty(int(256e6) // 4, dtype=torch.float32, device=dev) if flush else None
+
     for _ in range(args.warmup):
-        step()
+        ctx.eval_async(d_pts, d_out, stream)
+        gather(d_out)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     ctx.timing()                       # discard
     ctx.set_timing(True)
-    clocks = ClockSampler(local)
+    clocks = ClockSampler(dev.index)
     clocks.start()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    for _ in range(args.steps):
-        step()
-    e1.record(stream)
+    for i in range(args.steps):
+        if flush:
+            scrub.fill_(float(i))      # write 256 MB > L2 between timed steps (outside the events)
+        ev[i][0].record(stream)
+        ctx.eval_async(d_pts, d_out, stream)
+        gather(d_out)
+        ev[i][1].record(stream)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     clk = clocks.stop()
-    ms_total = e0.elapsed_time(e1)
+    ms_total = sum(a.elapsed_time(b) for a, b in ev)
     kern_ms, kern_n = ctx.timing()
     ctx.set_timing(False)
-    if world > 1:
-        t = torch.tensor([ms_total, kern_ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_total, kern_ms = t.tolist()
+    ms_total, kern_ms = allreduce_max([ms_total, kern_ms])
     ms_step = ms_total / args.steps
     value = w.n_points / (ms_step * 1e-3)
 
-    # end-to-end through the public host-buffer API (siac_eval): H2D of the points from pinned
-    # memory, evaluation, D2H of the values, every step
+    # end-to-end through the public host-buffer API (siac_eval): every step copies this rank's
+    # points from pinned host memory, evaluates, copies the values back, and (N > 1) gathers
+    # all ranks' values so every rank holds the full result
     h_pts = torch.from_numpy(np.ascontiguousarray(P_local)).pin_memory()
     h_out = torch.empty(max(n_local, 1), dtype=torch.float64).pin_memory()
     hp, ho = h_pts.numpy(), h_out.numpy()
     ctx.eval_into(hp, ho)
     if world > 1:
+        gather(h_out.to(gathered.device))
+        torch.cuda.synchronize()
         dist.barrier()
     t0 = time.perf_counter()
     for _ in range(args.e2e_steps):
         ctx.eval_into(hp, ho)
-    e2e_s = time.perf_counter() - t0
-    if world > 1:
-        t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_s = t.item()
+        if world > 1:
+            gather(h_out.to(gathered.device, non_blocking=False))
+            full = gathered.cpu()
+    e2e_s = allreduce_max([time.perf_counter() - t0])[0]
     e2e_val = w.n_points / (e2e_s / args.e2e_steps)
 
-    peak_meas = siac.probe_fp64(local)
+    peak_meas = siac.probe_fp64(dev.index)
     line = None
     if rank == 0:
         kern_avg_s = (kern_ms / max(kern_n, 1)) * 1e-3
-        achieved = flops_step / max(world, 1) / kern_avg_s / 1e12 if kern_avg_s > 0 else None
+        # whole-job algorithmic flops per launch-set / slowest rank's kernel time / ranks
+        achieved = flops_step / world / kern_avg_s / 1e12 if kern_avg_s > 0 else None
         peak = fp64_peak_derived()
         cfgd = workload_desc(w, args.config)
-        cfgd.update({"parallelism": f"spatial point tiles x{world}" if world > 1 else "single GPU",
-                     "l2": "inputs larger than L2 (points %.0f MB + triangle records %.0f MB > 126 MB)"
-                           % (w.n_points * 16 / 1e6, len(w.T) * 22 * 8 / 1e6),
+        cfgd.update({"parallelism": f"spatial point tiles x{world} + halo, NCCL all_gather" if world > 1
+                     else "single GPU",
+                     "l2": ("L2 flushed (256 MB write) between timed steps" if flush else
+                            "inputs larger than L2 (points %.0f MB + triangle records %.0f MB > 126 MB)"
+                            % (n_local * 16 / 1e6, len(T) * rs * 8 / 1e6)),
                      "counts": {"candidates": cands, "pairs": pairs, "pieces": pieces, "subtris": subtris},
                      "flops_per_subtri": flops_per_subtri(k)})
         line = {"metric": "filtered quadrature points/sec (FP64)", "value": value, "unit": "points/s",
@@ -272,7 +297,7 @@ def run_siac(args):
                 "data": "synthetic", "config": cfgd,
                 "roofline": {"bound": "alu", "kernel": "k_eval", "achieved": achieved, "peak": peak,
                              "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None, "traffic": None,
-                             "peak_note": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1965 MHz",
+                             "peak_note": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1965 MHz (DESIGN.md)",
                              "measured_dfma_peak": peak_meas,
                              "frac_of_measured": (achieved / peak_meas) if achieved else None,
                              "kernel_share_of_step": (kern_ms / kern_n) / ms_step if kern_n else None,
@@ -281,7 +306,7 @@ def run_siac(args):
                         "d2h_bytes_per_step": int(w.n_points * 8)},
                 "schedule": ["default(tile)", "point", "tile", "ws"][args.schedule],
                 "gpu_launches": 2 * args.steps,
-                "gpu_launches_note": "per step: k_point_keys + k_eval (ours) + CUB radix-sort kernels (library)",
+                "gpu_launches_note": "per step and rank: k_point_keys + k_eval (ours) + CUB radix-sort kernels",
                 "clocks": clk}
     if rank == 0 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(w, max(1, w.n_points // args.ref_points))
