@@ -274,7 +274,7 @@ def run_siac(args):
             gather(h_out.to(gathered.device, non_blocking=False))
             full = gathered.cpu()
     e2e_s = allreduce_max([time.perf_counter() - t0])[0]
-    e2e_val = w.n_points / (e2e_s / args.e2e_steps)
+    e2e_val = w.n_points / (e2e_s / args.e2e_steps) if args.e2e_steps > 0 else None
 
     peak_meas = siac.probe_fp64(dev.index)
     line = None
