@@ -64,8 +64,12 @@ typedef struct {        /* geometry counts of the last evaluation (see siac_set_
     int64_t n_points;
     int64_t candidates; /* (point, triangle image) bounding-box tests */
     int64_t pairs;      /* (point, triangle image) pairs whose boxes overlap */
-    int64_t pieces;     /* non-empty clipped polygons (triangle image ∩ kernel cell) */
-    int64_t subtris;    /* fan sub-triangles integrated = sum over pieces of (vertices - 2) */
+    int64_t pieces;     /* non-empty clipped polygons (triangle image ∩ kernel cell) integrated
+                           piece by piece (schedules POINT/TILE/WS; JUMP: general-path pairs only) */
+    int64_t subtris;    /* fan sub-triangles of those pieces = sum over pieces of (vertices - 2) */
+    int64_t corner_terms;  /* JUMP: closed-form corner terms (one per pair and axis with a knot) */
+    int64_t cross_terms;   /* JUMP: pairs with a knot on both axes (clipped corner-corner terms) */
+    int64_t cross_subtris; /* JUMP: fan sub-triangles integrated for the cross terms */
 } siac_counters;
 
 /*
@@ -111,19 +115,27 @@ siac_status siac_eval(siac_ctx *ctx, const double *points_xy, int64_t n_points, 
 siac_status siac_eval_async(siac_ctx *ctx, const double *d_points_xy, int64_t n_points,
                             double *d_values_out, void *cuda_stream);
 
-/* Evaluation schedule (same result up to summation order):
- *   SIAC_SCHEDULE_DEFAULT (0) the fastest measured schedule (currently SIAC_SCHEDULE_TILE);
+/* Evaluation schedule (same result up to rounding):
+ *   SIAC_SCHEDULE_DEFAULT (0) the fastest measured schedule (currently SIAC_SCHEDULE_JUMP);
  *   SIAC_SCHEDULE_POINT   (1) one thread per point, clip and integrate inline (the paper's
  *                         per-point evaluation, Alg. 2, one thread per point);
  *   SIAC_SCHEDULE_TILE    (2) one warp per tile of 32 Morton-ordered points: ballot-compacted
  *                         candidate tests, register-only Sutherland-Hodgman splits, sub-triangles
  *                         staged in shared memory and integrated 32 at a time by the full warp;
  *   SIAC_SCHEDULE_WS      (3) persistent warp-specialized variant of TILE: producer warps clip,
- *                         paired consumer warps integrate double-buffered batches (mbarriers). */
+ *                         paired consumer warps integrate double-buffered batches (mbarriers);
+ *   SIAC_SCHEDULE_JUMP    (4) the same exact decomposition (Eq. (2)) reorganised with the spline
+ *                         jumps of K: K = base cell polynomial + alpha (t - X)^k on the triangle's
+ *                         one-vertex side of a knot X, so each pair is the whole-triangle moment
+ *                         term + closed-form corner polynomials (precomputed per triangle at
+ *                         create time) + one clipped corner-corner piece integrated by quadrature
+ *                         when both axes have a knot (csrc/siac_jump.cuh).  Pairs with two knots
+ *                         on an axis (h < triangle size) use the clip-and-integrate path. */
 #define SIAC_SCHEDULE_DEFAULT 0
 #define SIAC_SCHEDULE_POINT 1
 #define SIAC_SCHEDULE_TILE 2
 #define SIAC_SCHEDULE_WS 3
+#define SIAC_SCHEDULE_JUMP 4
 siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule);
 
 /* Enable (1) / disable (0) geometry counting in later evaluations (adds atomics; off by default). */

@@ -24,6 +24,7 @@
 #include "siac_device.cuh"
 #include "siac_tile.cuh"
 #include "siac_ws.cuh"
+#include "siac_jump.cuh"
 #include "siac_math.h"
 
 #define SIAC_VERSION "siac-b200 0.1 (sm_100a, fp64)"
@@ -43,6 +44,7 @@ struct siac_ctx {
     double ex = 0, ey = 0;       // max triangle bbox extents
     // device mesh
     double *d_rec = nullptr;
+    double *d_jrec = nullptr;    // schedule JUMP records (siac_jump.cuh)
     double4 *d_bbox = nullptr;
     int *d_cell_start = nullptr;
     double *d_kc = nullptr;
@@ -55,7 +57,7 @@ struct siac_ctx {
     int64_t cap_host = 0;
     double *d_hpts = nullptr, *d_hout = nullptr;
     // counters
-    int schedule = 0;            // 0 = default (= 2), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized
+    int schedule = 0;            // 0 = default (= 4), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump
     int *d_tile_counter = nullptr;
     int num_sms = 148;
     bool counting = false;
@@ -171,13 +173,14 @@ struct EvalArgs {
     int64_t np;
     double *out;
     const double *rec;
+    const double *jrec;
     const double4 *bbox;
     const int *cell_start;
     const double *kc;
     double x0, y0, Lx, Ly, h, inv_h, hw;   // hw = W/2 (physical)
     double cw, chh, ex, ey;
     int ncx, ncy, periodic;
-    unsigned long long *cnt;  // [candidates, pairs, pieces, subtris]
+    unsigned long long *cnt;  // [candidates, pairs, pieces, subtris, corner, cross, cross_subtris, -]
 };
 
 __device__ __forceinline__ uint32_t spread16(uint32_t v) {
@@ -289,7 +292,19 @@ __global__ void __launch_bounds__(128) k_eval_v1(EvalArgs a) {
 
 template <int K>
 void launch_eval(const EvalArgs &a, bool count, int schedule, int *tile_counter, int num_sms, cudaStream_t st) {
-    if (schedule == 0) schedule = 2;     // the default schedule
+    if (schedule == 0) schedule = 4;     // the default schedule
+    if (schedule == 4) {
+        siacjump::JumpArgs j;
+        j.pts = a.pts; j.perm = a.perm; j.np = a.np; j.out = a.out; j.rec = a.rec; j.jrec = a.jrec; j.bbox = a.bbox;
+        j.cell_start = a.cell_start; j.kc = a.kc; j.x0 = a.x0; j.y0 = a.y0; j.Lx = a.Lx; j.Ly = a.Ly;
+        j.inv_h = a.inv_h; j.hw = a.hw; j.cw = a.cw; j.chh = a.chh; j.ex = a.ex; j.ey = a.ey;
+        j.ncx = a.ncx; j.ncy = a.ncy; j.periodic = a.periodic; j.cnt = a.cnt;
+        const int64_t ntiles = (a.np + 31) / 32;
+        const unsigned grid = (unsigned)((ntiles + siacjump::WARPS - 1) / siacjump::WARPS);
+        if (count) siacjump::k_eval_jump<K, true><<<grid, siacjump::WARPS * 32, 0, st>>>(j);
+        else siacjump::k_eval_jump<K, false><<<grid, siacjump::WARPS * 32, 0, st>>>(j);
+        return;
+    }
     if (schedule == 3) {
         siacws::WsArgs w;
         w.pts = a.pts; w.perm = a.perm; w.np = a.np; w.out = a.out; w.rec = a.rec; w.bbox = a.bbox;
@@ -371,13 +386,13 @@ void eval_device(siac_ctx *c, const double *d_pts, int64_t np, double *d_out, cu
     CK(cub::DeviceRadixSort::SortPairs(c->d_cub, c->cub_bytes, kb, vb, (int)np, 0, 2 * end_bit, st));
     EvalArgs a;
     a.pts = d_pts; a.perm = vb.Current(); a.np = np; a.out = d_out;
-    a.rec = c->d_rec; a.bbox = c->d_bbox; a.cell_start = c->d_cell_start; a.kc = c->d_kc;
+    a.rec = c->d_rec; a.jrec = c->d_jrec; a.bbox = c->d_bbox; a.cell_start = c->d_cell_start; a.kc = c->d_kc;
     a.x0 = c->dom[0]; a.y0 = c->dom[1]; a.Lx = Lx; a.Ly = Ly;
     a.h = c->h; a.inv_h = c->inv_h; a.hw = 0.5 * (3 * c->k + 1) * c->h;
     a.cw = c->cw; a.chh = c->chh; a.ex = c->ex; a.ey = c->ey;
     a.ncx = c->ncx; a.ncy = c->ncy; a.periodic = c->periodic;
     a.cnt = c->d_cnt;
-    if (c->counting) CK(cudaMemsetAsync(c->d_cnt, 0, 4 * sizeof(unsigned long long), st));
+    if (c->counting) CK(cudaMemsetAsync(c->d_cnt, 0, 8 * sizeof(unsigned long long), st));
     cudaEvent_t ev_stop = nullptr;
     if (c->timing) {
         if (c->ev_used == c->ev.size()) {
@@ -421,7 +436,7 @@ void free_ctx(siac_ctx *c) {
     if (!c) return;
     cudaSetDevice(c->device);
     for (auto &e : c->ev) { cudaEventDestroy(e.first); cudaEventDestroy(e.second); }
-    void *ptrs[] = {c->d_rec, c->d_bbox, c->d_cell_start, c->d_kc, c->d_keys[0], c->d_keys[1],
+    void *ptrs[] = {c->d_rec, c->d_jrec, c->d_bbox, c->d_cell_start, c->d_kc, c->d_keys[0], c->d_keys[1],
                     c->d_idx[0], c->d_idx[1], c->d_cub, c->d_hpts, c->d_hout, c->d_cnt, c->d_tile_counter};
     for (void *p : ptrs)
         if (p) cudaFree(p);
@@ -526,10 +541,10 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
         std::vector<double> R = siac::dubiner_to_centred(k);
         CK(cudaMalloc(&c->d_kc, sizeof(double) * kc.size()));
         CK(cudaMemcpy(c->d_kc, kc.data(), sizeof(double) * kc.size(), cudaMemcpyHostToDevice));
-        CK(cudaMalloc(&c->d_cnt, 4 * sizeof(unsigned long long)));
+        CK(cudaMalloc(&c->d_cnt, 8 * sizeof(unsigned long long)));
         CK(cudaMalloc(&c->d_tile_counter, sizeof(int)));
         c->num_sms = prop.multiProcessorCount;
-        CK(cudaMemset(c->d_cnt, 0, 4 * sizeof(unsigned long long)));
+        CK(cudaMemset(c->d_cnt, 0, 8 * sizeof(unsigned long long)));
         const int64_t ncell = (int64_t)c->ncx * c->ncy;
         CK(cudaMalloc(&c->d_cell_start, sizeof(int) * (ncell + 1)));
         if (nt == 0) {
@@ -578,6 +593,22 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
             k_gather<<<nblk(nt, 256), 256>>>(rec_u, bb_u, vb.Current(), nt, rs, c->d_rec, c->d_bbox);
             CK(cudaGetLastError());
             k_cell_start<<<nblk(ncell + 1, 256), 256>>>(kb.Current(), nt, ncell, c->d_cell_start);
+            CK(cudaGetLastError());
+            // schedule JUMP: per-triangle moments and corner polynomials (siac_jump.cuh)
+            int jrs = 0;
+            switch (k) {
+                case 1: jrs = siacjump::JRec<1>::RS; break;
+                case 2: jrs = siacjump::JRec<2>::RS; break;
+                case 3: jrs = siacjump::JRec<3>::RS; break;
+                default: jrs = siacjump::JRec<4>::RS; break;
+            }
+            CK(cudaMalloc(&c->d_jrec, sizeof(double) * jrs * nt));
+            switch (k) {
+                case 1: siacjump::k_prep_jump<1><<<nblk(nt, 128), 128>>>(c->d_rec, nt, p->h, c->d_jrec); break;
+                case 2: siacjump::k_prep_jump<2><<<nblk(nt, 128), 128>>>(c->d_rec, nt, p->h, c->d_jrec); break;
+                case 3: siacjump::k_prep_jump<3><<<nblk(nt, 128), 128>>>(c->d_rec, nt, p->h, c->d_jrec); break;
+                default: siacjump::k_prep_jump<4><<<nblk(nt, 128), 128>>>(c->d_rec, nt, p->h, c->d_jrec); break;
+            }
             CK(cudaGetLastError());
             CK(cudaDeviceSynchronize());
         } catch (...) {
@@ -638,7 +669,7 @@ siac_status siac_stats(siac_ctx *ctx, siac_counters *out) {
     if (!ctx || !out) { g_err = "NULL argument"; return SIAC_EINVAL; }
     return run_guarded(&ctx->err, [&]() {
         CK(cudaSetDevice(ctx->device));
-        unsigned long long h[4];
+        unsigned long long h[8];
         CK(cudaDeviceSynchronize());
         CK(cudaMemcpy(h, ctx->d_cnt, sizeof(h), cudaMemcpyDeviceToHost));
         out->n_points = ctx->last_np;
@@ -646,12 +677,15 @@ siac_status siac_stats(siac_ctx *ctx, siac_counters *out) {
         out->pairs = (int64_t)h[1];
         out->pieces = (int64_t)h[2];
         out->subtris = (int64_t)h[3];
+        out->corner_terms = (int64_t)h[4];
+        out->cross_terms = (int64_t)h[5];
+        out->cross_subtris = (int64_t)h[6];
     });
 }
 
 siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule) {
     if (!ctx) { g_err = "NULL context"; return SIAC_EINVAL; }
-    if (schedule < 0 || schedule > 3) { ctx->err = "unknown schedule"; return SIAC_EINVAL; }
+    if (schedule < 0 || schedule > 4) { ctx->err = "unknown schedule"; return SIAC_EINVAL; }
     ctx->schedule = schedule;
     return SIAC_OK;
 }

@@ -1,0 +1,590 @@
+// siac_jump.cuh -- schedule JUMP (the default): the exact decomposition of Eq. (2) reorganised
+// around the spline structure of the kernel, so that almost no per-pair quadrature is needed.
+//
+// Why it is exact.  K is a spline of degree k on the unit knots t_m = T0 + m (m = 0..3k+1,
+// T0 = -(3k+1)/2), C^{k-1} everywhere and zero outside [t_0, t_{3k+1}] (PAPER.md L196-208,
+// L250-254).  Across a knot only the k-th derivative jumps, so with P_i the polynomial of K on
+// cell i (P_{-1} = P_{3k+1} = 0)
+//     P_m(t) - P_{m-1}(t) = alpha_m (t - t_m)^k,   alpha_m = lead(P_m) - lead(P_{m-1}).
+// When h >= the longest edge (the paper's h = s, L430/L440), a triangle's x-range (in z = (y-x)/h
+// units) is <= 1, so at most one knot X lies strictly inside it, and on the triangle
+//     K(z1) = B1(z1) + C1(z1),  B1 = P_{base},  C1 = sgn alpha_X (z1 - X)^k 1[corner_x],
+// where corner_x = T ∩ {z1 on the side of X holding a single vertex} is a triangle: the
+// Sutherland-Hodgman clip (Alg. 1) of T against the line z1 = X, on the "alone vertex" side
+// (base = the cell on the other side; sgn = +1 if the corner is right of X, -1 if left).
+// Likewise for z2.  Eq. (2)'s integral over the pieces of T then splits into four terms:
+//     I00 = \int_T B1 B2 u                    -- per-triangle moments mu_ab = \int_T zeta1^a zeta2^b u
+//     I10 = \int_{corner_x} C1 B2 u           -- corner_x is the homothetic image of a fixed
+//     I01 = \int_{corner_y} B1 C2 u              reference corner about the alone vertex, ratio
+//                                                lambda, so \int_{corner} (zeta1 - X)^k zeta2^b u
+//                                                = lambda^{k+2} G_b(lambda), G_b a polynomial of
+//                                                degree k+b precomputed per triangle at create time
+//     I11 = \int_{corner_x ∩ corner_y} C1 C2 u -- corner_x clipped by the line z2 = Y (SH), fan-
+//                                                triangulated, degree-3k Gauss quadrature.
+// zeta = (y - centroid)/h is the per-triangle frame the precomputed data live in; z = zeta +
+// delta, delta = (centroid + image shift - x)/h.  Pairs with two or more knots inside a range
+// (only when h is smaller than the triangles) take the general per-pair path of siac_device.cuh.
+//
+// Execution: one warp per tile of 32 Morton-consecutive points (lane = point), exactly like
+// schedule TILE for candidate search; for every candidate triangle the whole warp evaluates the
+// closed-form terms with warp-uniform record loads (one triangle, 32 stencils), and the rare I11
+// terms are queued in shared memory and integrated 32 at a time by the full warp.
+#pragma once
+
+#include "siac_device.cuh"
+
+namespace siacjump {
+
+using namespace siacdev;
+
+// ------------------------------------------------------------------ jump record layout (doubles)
+//   [0,1]              centroid (physical)
+//   [2..6] / [7..11]   axis x / y: zlo, zmid, zhi (sorted vertex coords, zeta frame),
+//                      invL = 1/(zmid-zlo), invR = 1/(zhi-zmid)  (0 if that corner is degenerate)
+//   [OFF_MU ..]        mu[a*(K+1)+b] = \int_T zeta1^a zeta2^b u dzeta, a, b = 0..K
+//   [OFF_G ..]         4 corners (x-right, x-left, y-top, y-bottom) x NG coefficients:
+//                      block b (= power of the other coordinate, 0..K) holds G_b[0..K+b]
+//   [OFF_GEO ..]       per axis: L, Mv, R (vertices sorted by that coordinate), C' (the point of
+//                      edge L-R at coordinate Mv) -- 8 doubles per axis
+//   [OFF_MAP ..]       rho = m00 z1 + m01 z2 + r0, sigma = m10 z1 + m11 z2 + s0 (centred reference
+//                      coordinates of the record's modes, rho = 3r-1, sigma = 3s-1)
+//   [OFF_D ..]         modes d in centred monomials, Horner order (siac_device.cuh, Rec<K>)
+template <int K> struct JRec {
+    static constexpr int NB = (K + 1) * (K + 2) / 2;
+    static constexpr int NG = (K + 1) * (3 * K + 2) / 2;
+    static constexpr int OFF_AX = 2;
+    static constexpr int OFF_MU = 12;
+    static constexpr int OFF_G = OFF_MU + (K + 1) * (K + 1);
+    static constexpr int OFF_GEO = OFF_G + 4 * NG;
+    static constexpr int OFF_MAP = OFF_GEO + 16;
+    static constexpr int OFF_D = OFF_MAP + 6;
+    static constexpr int RAW = OFF_D + NB;
+    static constexpr int RS = (RAW + 1) & ~1;
+};
+__host__ __device__ constexpr int g_off(int K, int b) { return b * (K + 1) + b * (b - 1) / 2; }
+
+// ------------------------------------------------------------------ create-time record build
+
+// polynomial in lambda (degree <= D, coefficients p[0..D]) times (c0 + c1 lambda)
+template <int D> __device__ __forceinline__ void pmul_lin(double *p, int deg, double c0, double c1) {
+    p[deg + 1 < D + 1 ? deg + 1 : D] = 0.0;
+    for (int j = deg + 1; j >= 1; --j) p[j] = fma(p[j], c0, p[j - 1] * c1);
+    p[0] *= c0;
+}
+
+// coefficients in lambda of u(A + lambda d), u = horner2(dm, rho, sigma), rho/sigma affine
+template <int K>
+__device__ void u_along(const double *dm, double rA, double rD, double sA, double sD, double *ul) {
+    double in[K + 2];
+    int off = 0;
+    for (int j = 0; j <= K; ++j) ul[j] = 0.0;
+    int udeg = 0;
+    for (int a = K; a >= 0; --a) {
+        const int n = K - a;
+        for (int j = 0; j <= K + 1; ++j) in[j] = 0.0;
+        in[0] = dm[off + n];
+        int deg = 0;
+        for (int b = n - 1; b >= 0; --b) {
+            pmul_lin<K + 1>(in, deg, sA, sD);
+            ++deg;
+            in[0] += dm[off + b];
+        }
+        if (a == K) {
+            for (int j = 0; j <= deg; ++j) ul[j] = in[j];
+            udeg = deg;
+        } else {
+            double t[K + 2];
+            for (int j = 0; j <= K + 1; ++j) t[j] = j <= K ? ul[j] : 0.0;
+            pmul_lin<K + 1>(t, udeg, rA, rD);
+            udeg = udeg + 1 > deg ? udeg + 1 : deg;
+            for (int j = 0; j <= K; ++j) ul[j] = t[j] + (j <= deg ? in[j] : 0.0);
+        }
+        off += n + 1;
+    }
+}
+
+// One thread per triangle (binning order).  rec: siacdev::Rec<K> records (same order).
+template <int K>
+__global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jrec) {
+    using R = Rec<K>;
+    using J = JRec<K>;
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= nt) return;
+    const double *r = rec + (int64_t)R::RS * t;
+    double *o = jrec + (int64_t)J::RS * t;
+    const double inv_h = 1.0 / h;
+    const double cx = (r[0] + r[2] + r[4]) / 3.0, cy = (r[1] + r[3] + r[5]) / 3.0;
+    double zx[3], zy[3];
+    for (int v = 0; v < 3; ++v) { zx[v] = (r[2 * v] - cx) * inv_h; zy[v] = (r[2 * v + 1] - cy) * inv_h; }
+    // (rho, sigma) = M (z - z_v0) - (1, 1), M = 3 h A^{-1}: affine in zeta
+    const double m00 = r[6], m01 = r[7], m10 = r[8], m11 = r[9];
+    const double r0 = -fma(m00, zx[0], m01 * zy[0]) - 1.0, s0 = -fma(m10, zx[0], m11 * zy[0]) - 1.0;
+    double dm[R::NB];
+    for (int j = 0; j < R::NB; ++j) dm[j] = r[R::OFF_D + j];
+    o[0] = cx; o[1] = cy;
+    // moments over T
+    {
+        const double e1x = zx[1] - zx[0], e1y = zy[1] - zy[0], e2x = zx[2] - zx[0], e2y = zy[2] - zy[0];
+        const double area = 0.5 * fabs(e1x * e2y - e1y * e2x);
+        double mu[(K + 1) * (K + 1)];
+        for (int i = 0; i < (K + 1) * (K + 1); ++i) mu[i] = 0.0;
+        for (int q = 0; q < Rule<K>::NQ; ++q) {
+            const double a1 = zx[0] + qr<K>(q) * e1x + qs<K>(q) * e2x;
+            const double a2 = zy[0] + qr<K>(q) * e1y + qs<K>(q) * e2y;
+            const double u = horner2<K>(dm, fma(m00, a1, fma(m01, a2, r0)), fma(m10, a1, fma(m11, a2, s0)));
+            double pa = area * qw<K>(q) * u;
+            for (int a = 0; a <= K; ++a) {
+                double pb = pa;
+                for (int b = 0; b <= K; ++b) { mu[a * (K + 1) + b] += pb; pb *= a2; }
+                pa *= a1;
+            }
+        }
+        for (int i = 0; i < (K + 1) * (K + 1); ++i) o[J::OFF_MU + i] = mu[i];
+    }
+    for (int ax = 0; ax < 2; ++ax) {
+        const double *cA = ax == 0 ? zx : zy;   // coordinate along the cut axis
+        int iL = 0, iM = 1, iR = 2;
+        if (cA[iL] > cA[iM]) { int s = iL; iL = iM; iM = s; }
+        if (cA[iM] > cA[iR]) { int s = iM; iM = iR; iR = s; }
+        if (cA[iL] > cA[iM]) { int s = iL; iL = iM; iM = s; }
+        const double Lx = zx[iL], Ly = zy[iL], Mx = zx[iM], My = zy[iM], Rx = zx[iR], Ry = zy[iR];
+        const double lo = cA[iL], mid = cA[iM], hi = cA[iR];
+        const double f = (mid - lo) / (hi - lo);
+        const double Cx = Lx + f * (Rx - Lx), Cy = Ly + f * (Ry - Ly);
+        double *ad = o + J::OFF_AX + 5 * ax;
+        ad[0] = lo; ad[1] = mid; ad[2] = hi;
+        ad[3] = mid > lo ? 1.0 / (mid - lo) : 0.0;
+        ad[4] = hi > mid ? 1.0 / (hi - mid) : 0.0;
+        double *geo = o + J::OFF_GEO + 8 * ax;
+        geo[0] = Lx; geo[1] = Ly; geo[2] = Mx; geo[3] = My; geo[4] = Rx; geo[5] = Ry; geo[6] = Cx; geo[7] = Cy;
+        for (int side = 0; side < 2; ++side) {      // 0: apex = R (right/top), 1: apex = L
+            const double Ax = side == 0 ? Rx : Lx, Ay = side == 0 ? Ry : Ly;
+            const double e1x = Mx - Ax, e1y = My - Ay, e2x = Cx - Ax, e2y = Cy - Ay;
+            const double area = 0.5 * fabs(e1x * e2y - e1y * e2x);
+            double g[J::NG];
+            for (int i = 0; i < J::NG; ++i) g[i] = 0.0;
+            const double rA = fma(m00, Ax, fma(m01, Ay, r0)), sA = fma(m10, Ax, fma(m11, Ay, s0));
+            const double aO = ax == 0 ? Ay : Ax;
+            for (int q = 0; q < Rule<K>::NQ; ++q) {
+                const double dx = qr<K>(q) * e1x + qs<K>(q) * e2x, dy = qr<K>(q) * e1y + qs<K>(q) * e2y;
+                const double xiA = (ax == 0 ? Ax + dx : Ay + dy) - mid;   // (xi_axis - Mv_axis)
+                double wq = area * qw<K>(q);
+                for (int i = 0; i < K; ++i) wq *= xiA;
+                double ul[K + 1];
+                u_along<K>(dm, rA, fma(m00, dx, m01 * dy), sA, fma(m10, dx, m11 * dy), ul);
+                double w[2 * K + 2];
+                for (int j = 0; j < 2 * K + 2; ++j) w[j] = j <= K ? ul[j] : 0.0;
+                const double dO = ax == 0 ? dy : dx;
+                for (int b = 0; b <= K; ++b) {
+                    const int deg = K + b;
+                    double *gb = g + g_off(K, b);
+                    for (int j = 0; j <= deg; ++j) gb[j] = fma(wq, w[j], gb[j]);
+                    if (b < K) pmul_lin<2 * K + 1>(w, deg, aO, dO);
+                }
+            }
+            double *go = o + J::OFF_G + (2 * ax + side) * J::NG;
+            for (int i = 0; i < J::NG; ++i) go[i] = area > 0.0 ? g[i] : 0.0;
+        }
+    }
+    double *mp = o + J::OFF_MAP;
+    mp[0] = m00; mp[1] = m01; mp[2] = m10; mp[3] = m11; mp[4] = r0; mp[5] = s0;
+    for (int j = 0; j < R::NB; ++j) o[J::OFF_D + j] = dm[j];
+    for (int j = J::RAW; j < J::RS; ++j) o[j] = 0.0;
+}
+
+// ------------------------------------------------------------------ evaluation
+
+#ifndef SIAC_JUMP_WARPS
+#define SIAC_JUMP_WARPS 4
+#endif
+#ifndef SIAC_JUMP_MINB
+#define SIAC_JUMP_MINB 4
+#endif
+constexpr int WARPS = SIAC_JUMP_WARPS;
+constexpr int QCAP = 64;      // cross-term queue: < 32 left over + 32 new
+
+struct WarpSmem {
+    int qtri[QCAP];
+    int qinfo[QCAP];          // lane | sx << 5 | sy << 6 | mx << 7 | my << 12
+    double qX[QCAP], qY[QCAP];
+    double acc[32];
+    double4 cbox[32];
+    double px[32], py[32];
+};
+
+struct JumpArgs {
+    const double *pts;
+    const int *perm;
+    int64_t np;
+    double *out;
+    const double *rec;        // Rec<K> (general fallback)
+    const double *jrec;       // JRec<K>
+    const double4 *bbox;
+    const int *cell_start;
+    const double *kc;
+    double x0, y0, Lx, Ly, inv_h, hw;
+    double cw, chh, ex, ey;
+    int ncx, ncy, periodic;
+    unsigned long long *cnt;  // candidates, pairs, pieces, subtris, corner, cross, cross_subtris
+};
+
+struct Cut {
+    int state;     // 0 none, 1 one knot, 2 several knots (general path)
+    int base;      // base cell (may be outside 0..NC-1: zero polynomial)
+    int side;      // 0: corner on the high side (apex = max vertex), 1: low side
+    int m;         // knot index
+    double X;      // knot position in the zeta frame
+    double lam;    // homothety ratio of the corner
+};
+
+template <int K>
+__device__ __forceinline__ Cut axis_cut(const double *ad, double dl) {
+    constexpr int NC = 3 * K + 1;
+    constexpr double T0 = -0.5 * (3 * K + 1);
+    const double zlo = __ldg(ad + 0), zmid = __ldg(ad + 1), zhi = __ldg(ad + 2);
+    const double lo = (zlo + dl) - T0, hi = (zhi + dl) - T0;
+    const double fl = floor(lo);
+    const int m1 = max((int)fl + 1, 0), m2 = min((int)ceil(hi) - 1, NC);
+    Cut c;
+    c.state = m2 < m1 ? 0 : (m2 == m1 ? 1 : 2);
+    c.m = m1;
+    c.X = (T0 + m1) - dl;
+    c.base = (int)fl;
+    c.side = 0;
+    c.lam = 0.0;
+    if (c.state == 1) {
+        if (c.X > zmid) { c.side = 0; c.base = m1 - 1; c.lam = (zhi - c.X) * __ldg(ad + 4); }
+        else { c.side = 1; c.base = m1; c.lam = (c.X - zlo) * __ldg(ad + 3); }
+    }
+    return c;
+}
+
+// Taylor coefficients p_a (a = 0..K) of P_base(zeta + dl) in powers of zeta.  kcp: padded cell
+// table, row i+1 = cell i, rows 0 and NC+1 zero.
+template <int K>
+__device__ __forceinline__ void base_taylor(const double *kcp, int base, double dl, double *p) {
+    constexpr int NC = 3 * K + 1;
+    constexpr double T0 = -0.5 * (3 * K + 1);
+    const int row = (base < 0 || base >= NC) ? 0 : base + 1;
+    const double e = dl - (T0 + base + 0.5);
+#pragma unroll
+    for (int j = 0; j <= K; ++j) p[j] = kcp[row * (K + 1) + j];
+#pragma unroll
+    for (int i = 0; i < K; ++i)
+#pragma unroll
+        for (int j = K - 1; j >= i; --j) p[j] = fma(e, p[j + 1], p[j]);
+}
+
+// lambda^{K+2} sum_b c_b G_b(lambda), G_b of degree K + b
+template <int K>
+__device__ __forceinline__ double corner_eval(const double *G, const double *c, double lam) {
+    double s = 0.0;
+#pragma unroll
+    for (int b = K; b >= 0; --b) {
+        const double *gb = G + g_off(K, b);
+        double v = __ldg(gb + K + b);
+#pragma unroll
+        for (int j = K + b - 1; j >= 0; --j) v = fma(v, lam, __ldg(gb + j));
+        s = fma(c[b], v, s);
+    }
+    double l2 = lam * lam, lp = l2;
+#pragma unroll
+    for (int i = 0; i < K; ++i) lp *= lam;
+    return lp * s;
+}
+
+// \int over triangle (p0, p1, p2) of (z1 - X)^K (z2 - Y)^K u(z), rule exact for degree 3K
+template <int K>
+__device__ __forceinline__ double integrate_cross(double p0x, double p0y, double p1x, double p1y, double p2x,
+                                                  double p2y, double X, double Y, const double *mp,
+                                                  const double *d) {
+    const double e1x = p1x - p0x, e1y = p1y - p0y, e2x = p2x - p0x, e2y = p2y - p0y;
+    const double area = 0.5 * fabs(e1x * e2y - e1y * e2x);
+    const double tx0 = p0x - X, ty0 = p0y - Y;
+    const double r0 = fma(mp[0], p0x, fma(mp[1], p0y, mp[4]));
+    const double rr = fma(mp[0], e1x, mp[1] * e1y), rs = fma(mp[0], e2x, mp[1] * e2y);
+    const double s0 = fma(mp[2], p0x, fma(mp[3], p0y, mp[5]));
+    const double sr = fma(mp[2], e1x, mp[3] * e1y), ss = fma(mp[2], e2x, mp[3] * e2y);
+    double acc = 0.0;
+#pragma unroll
+    for (int q = 0; q < Rule<K>::NQ; ++q) {
+        const double r = qr<K>(q), s = qs<K>(q);
+        const double tx = fma(e2x, s, fma(e1x, r, tx0));
+        const double ty = fma(e2y, s, fma(e1y, r, ty0));
+        const double rho = fma(rs, s, fma(rr, r, r0));
+        const double sig = fma(ss, s, fma(sr, r, s0));
+        const double t = tx * ty;
+        double tp = t;
+#pragma unroll
+        for (int i = 1; i < K; ++i) tp *= t;
+        acc = fma(qw<K>(q), tp * horner2<K>(d, rho, sig), acc);
+    }
+    return area * acc;
+}
+
+// Clip-and-integrate path for a pair with two or more knots inside an axis range (only when h is
+// smaller than the triangle): SH pieces + fan + quadrature (siac_device.cuh).  Out of line so its
+// polygon buffers do not burden the hot loop's registers.
+struct GenOut {
+    double v;
+    unsigned pieces, subtris;
+};
+template <int K, bool COUNT>
+__device__ __noinline__ GenOut general_pair(const double *__restrict__ rec, const double *kcp, int tri, double rsx,
+                                            double rsy, double x1, double x2, double inv_h) {
+    const double *rc = rec + (int64_t)Rec<K>::RS * tri;
+    double zx[3], zy[3];
+#pragma unroll
+    for (int v = 0; v < 3; ++v) {
+        zx[v] = ((__ldg(rc + 2 * v) + rsx) - x1) * inv_h;
+        zy[v] = ((__ldg(rc + 2 * v + 1) + rsy) - x2) * inv_h;
+    }
+    PairGeom g;
+    g.M00 = __ldg(rc + 6); g.M01 = __ldg(rc + 7); g.M10 = __ldg(rc + 8); g.M11 = __ldg(rc + 9);
+    g.zv0x = zx[0]; g.zv0y = zy[0];
+    double d[Rec<K>::NB];
+#pragma unroll
+    for (int m = 0; m < Rec<K>::NB; ++m) d[m] = __ldg(rc + Rec<K>::OFF_D + m);
+    Counts cn = {0, 0, 0};
+    GenOut o;
+    o.v = pair_contrib<K, COUNT>(zx, zy, kcp + (K + 1), d, g, cn);
+    o.pieces = (unsigned)cn.pieces;
+    o.subtris = (unsigned)cn.subtris;
+    return o;
+}
+
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+// Sum v over lanes with equal key (keys >= 32 ignored), in lane order, into S.acc[key].
+__device__ __forceinline__ void seg_add(WarpSmem &S, int key, double v, int lane) {
+    const unsigned grp = __match_any_sync(0xffffffffu, key);
+    const int leader = __ffs(grp) - 1;
+    double sum = (lane == leader) ? v : 0.0;
+    unsigned rest = grp & ~(1u << leader);
+    while (__any_sync(0xffffffffu, rest != 0)) {
+        const int src = rest ? __ffs(rest) - 1 : lane;
+        const double w = __shfl_sync(0xffffffffu, v, src);
+        if (rest) { if (lane == leader) sum += w; rest &= rest - 1; }
+    }
+    if (lane == leader && key < 32) S.acc[key] += sum;
+    __syncwarp();
+}
+
+// Integrate `take` queued cross terms (from the top of the queue), one per lane.
+template <int K, bool COUNT>
+__device__ __forceinline__ void drain(const JumpArgs &a, WarpSmem &S, const double *alpha, int &nq, int lane,
+                                      unsigned long long &c_xsub) {
+    using J = JRec<K>;
+    const int take = min(nq, 32);
+    int key = 32 + lane;
+    double v = 0.0;
+    if (lane < take) {
+        const int e = nq - 1 - lane;
+        const int tri = S.qtri[e], info = S.qinfo[e];
+        const double X = S.qX[e], Y = S.qY[e];
+        key = info & 31;
+        const int sx = (info >> 5) & 1, sy = (info >> 6) & 1, mx = (info >> 7) & 31, my = (info >> 12) & 31;
+        const double *jr = a.jrec + (int64_t)J::RS * tri;
+        const double *ad = jr + J::OFF_AX;
+        const double lam = sx == 0 ? (__ldg(ad + 2) - X) * __ldg(ad + 4) : (X - __ldg(ad + 0)) * __ldg(ad + 3);
+        const double *geo = jr + J::OFF_GEO;
+        const double Ax = __ldg(geo + (sx == 0 ? 4 : 0)), Ay = __ldg(geo + (sx == 0 ? 5 : 1));
+        const double p1x = fma(lam, __ldg(geo + 2) - Ax, Ax), p1y = fma(lam, __ldg(geo + 3) - Ay, Ay);
+        const double p2x = fma(lam, __ldg(geo + 6) - Ax, Ax), p2y = fma(lam, __ldg(geo + 7) - Ay, Ay);
+        // Sutherland-Hodgman clip of (A, P1, P2) by z2 = Y, keeping the y-corner's side
+        const double sgn = sy == 0 ? 1.0 : -1.0;
+        const double vx[3] = {Ax, p1x, p2x}, vy[3] = {Ay, p1y, p2y};
+        double ox[4], oy[4];
+        int n = 0;
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+            const int j = i == 2 ? 0 : i + 1;
+            const double di = sgn * (vy[i] - Y), dj = sgn * (vy[j] - Y);
+            if (di >= 0.0) { ox[n] = vx[i]; oy[n] = vy[i]; ++n; }
+            if ((di >= 0.0) != (dj >= 0.0)) {
+                const double t = (Y - vy[i]) / (vy[j] - vy[i]);
+                ox[n] = fma(t, vx[j] - vx[i], vx[i]); oy[n] = Y; ++n;
+            }
+        }
+        if (n >= 3) {
+            double mp[6], d[J::NB];
+#pragma unroll
+            for (int i = 0; i < 6; ++i) mp[i] = __ldg(jr + J::OFF_MAP + i);
+#pragma unroll
+            for (int i = 0; i < J::NB; ++i) d[i] = __ldg(jr + J::OFF_D + i);
+            v = integrate_cross<K>(ox[0], oy[0], ox[1], oy[1], ox[2], oy[2], X, Y, mp, d);
+            if (n == 4) v += integrate_cross<K>(ox[0], oy[0], ox[2], oy[2], ox[3], oy[3], X, Y, mp, d);
+            if (COUNT) c_xsub += n - 2;
+            const double cxf = sx == 0 ? alpha[mx] : -alpha[mx];
+            const double cyf = sy == 0 ? alpha[my] : -alpha[my];
+            v *= cxf * cyf;
+        }
+    }
+    nq -= take;
+    __syncwarp();
+    seg_add(S, key, v, lane);
+}
+
+template <int K, bool COUNT>
+__global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpArgs a) {
+    using J = JRec<K>;
+    constexpr int NC = 3 * K + 1;
+    __shared__ double kcp[(NC + 2) * (K + 1)];
+    __shared__ double alpha[NC + 1];
+    __shared__ WarpSmem wsm[WARPS];
+    for (int i = threadIdx.x; i < (NC + 2) * (K + 1); i += blockDim.x) {
+        const int row = i / (K + 1);
+        kcp[i] = (row == 0 || row == NC + 1) ? 0.0 : a.kc[i - (K + 1)];
+    }
+    __syncthreads();
+    for (int m = threadIdx.x; m <= NC; m += blockDim.x) alpha[m] = kcp[(m + 1) * (K + 1) + K] - kcp[m * (K + 1) + K];
+    __syncthreads();
+
+    const int lane = threadIdx.x & 31;
+    const int wid = threadIdx.x >> 5;
+    WarpSmem &S = wsm[wid];
+    const int64_t p0 = ((int64_t)blockIdx.x * WARPS + wid) * 32;
+    if (p0 >= a.np) return;                       // warp-uniform
+    const bool valid = p0 + lane < a.np;
+    int orig = -1;
+    double x1 = 0, x2 = 0;
+    if (valid) {
+        orig = a.perm[p0 + lane];
+        x1 = a.pts[2 * (int64_t)orig];
+        x2 = a.pts[2 * (int64_t)orig + 1];
+        if (a.periodic & 1) { x1 = x1 - a.Lx * floor((x1 - a.x0) / a.Lx); if (x1 >= a.x0 + a.Lx) x1 -= a.Lx; if (x1 < a.x0) x1 = a.x0; }
+        if (a.periodic & 2) { x2 = x2 - a.Ly * floor((x2 - a.y0) / a.Ly); if (x2 >= a.y0 + a.Ly) x2 -= a.Ly; if (x2 < a.y0) x2 = a.y0; }
+    }
+    S.px[lane] = x1;
+    S.py[lane] = x2;
+    S.acc[lane] = 0.0;
+    double tx0 = valid ? x1 : 1e300, tx1 = valid ? x1 : -1e300, ty0 = valid ? x2 : 1e300, ty1 = valid ? x2 : -1e300;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        tx0 = fmin(tx0, __shfl_xor_sync(0xffffffffu, tx0, o));
+        tx1 = fmax(tx1, __shfl_xor_sync(0xffffffffu, tx1, o));
+        ty0 = fmin(ty0, __shfl_xor_sync(0xffffffffu, ty0, o));
+        ty1 = fmax(ty1, __shfl_xor_sync(0xffffffffu, ty1, o));
+    }
+    const double sx0 = x1 - a.hw, sx1 = x1 + a.hw, sy0 = x2 - a.hw, sy1 = x2 + a.hw;     // own stencil
+    const double bx0 = tx0 - a.hw, bx1 = tx1 + a.hw, by0 = ty0 - a.hw, by1 = ty1 + a.hw;  // tile's stencils
+    int R0 = (int)floor((by0 - a.ey - a.y0) / a.chh) - 1, R1 = (int)floor((by1 - a.y0) / a.chh) + 1;
+    int C0 = (int)floor((bx0 - a.ex - a.x0) / a.cw) - 1, C1 = (int)floor((bx1 - a.x0) / a.cw) + 1;
+    if (!(a.periodic & 2)) { R0 = max(R0, 0); R1 = min(R1, a.ncy - 1); }
+    if (!(a.periodic & 1)) { C0 = max(C0, 0); C1 = min(C1, a.ncx - 1); }
+    __syncwarp();
+
+    double acc = 0.0;
+    int nq = 0;
+    unsigned long long c_cand = 0, c_pairs = 0, c_pieces = 0, c_sub = 0, c_corner = 0, c_cross = 0, c_xsub = 0;
+    for (int R = R0; R <= R1; ++R) {
+        int r = R, qy = 0;
+        if (a.periodic & 2) { r = ((R % a.ncy) + a.ncy) % a.ncy; qy = (R - r) / a.ncy; }
+        const double rsy = qy * a.Ly;
+        int C = C0;
+        while (C <= C1) {
+            int c = C, qx = 0;
+            if (a.periodic & 1) { c = ((C % a.ncx) + a.ncx) % a.ncx; qx = (C - c) / a.ncx; }
+            const int cend = (a.periodic & 1) ? min(C1, (qx + 1) * a.ncx - 1) : C1;
+            const double rsx = qx * a.Lx;
+            const int cb = c + (cend - C);
+            int t_cur = __ldg(a.cell_start + r * a.ncx + c);
+            const int t_end = __ldg(a.cell_start + r * a.ncx + cb + 1);
+            C = cend + 1;
+            for (; t_cur < t_end; t_cur += 32) {
+                const int n = min(32, t_end - t_cur);
+                bool keep = false;
+                if (lane < n) {
+                    double4 b = a.bbox[t_cur + lane];
+                    b.x += rsx; b.z += rsx; b.y += rsy; b.w += rsy;
+                    S.cbox[lane] = b;
+                    keep = (b.x < bx1 && b.z > bx0 && b.y < by1 && b.w > by0);
+                }
+                unsigned mask = __ballot_sync(0xffffffffu, keep);
+                __syncwarp();
+                while (mask) {
+                    const int j = __ffs(mask) - 1;
+                    mask &= mask - 1;
+                    const double4 b = S.cbox[j];
+                    const bool hit = valid && (b.x < sx1 && b.z > sx0 && b.y < sy1 && b.w > sy0);
+                    const unsigned hm = __ballot_sync(0xffffffffu, hit);
+                    if (COUNT) { c_cand += __popc(__ballot_sync(0xffffffffu, valid)); c_pairs += __popc(hm); }
+                    if (hm == 0) continue;
+                    const int tri = t_cur + j;
+                    const double *jr = a.jrec + (int64_t)J::RS * tri;
+                    bool cross = false;
+                    Cut cx, cy;
+                    if (hit) {
+                        const double dx = ((__ldg(jr + 0) + rsx) - x1) * a.inv_h;
+                        const double dy = ((__ldg(jr + 1) + rsy) - x2) * a.inv_h;
+                        cx = axis_cut<K>(jr + J::OFF_AX, dx);
+                        cy = axis_cut<K>(jr + J::OFF_AX + 5, dy);
+                        if (cx.state == 2 || cy.state == 2) {
+                            // general path: several knots inside a range (h < triangle size)
+                            const GenOut go = general_pair<K, COUNT>(a.rec, kcp, tri, rsx, rsy, x1, x2, a.inv_h);
+                            acc += go.v;
+                            if (COUNT) { c_pieces += go.pieces; c_sub += go.subtris; }
+                        } else {
+                            double p[K + 1], q[K + 1];
+                            base_taylor<K>(kcp, cx.base, dx, p);
+                            base_taylor<K>(kcp, cy.base, dy, q);
+                            double v = 0.0;
+#pragma unroll
+                            for (int aa = K; aa >= 0; --aa) {
+                                double s = 0.0;
+#pragma unroll
+                                for (int bb = K; bb >= 0; --bb) s = fma(q[bb], __ldg(jr + J::OFF_MU + aa * (K + 1) + bb), s);
+                                v = fma(p[aa], s, v);
+                            }
+                            if (cx.state) {
+                                const double cf = cx.side == 0 ? alpha[cx.m] : -alpha[cx.m];
+                                v = fma(cf, corner_eval<K>(jr + J::OFF_G + cx.side * J::NG, q, cx.lam), v);
+                            }
+                            if (cy.state) {
+                                const double cf = cy.side == 0 ? alpha[cy.m] : -alpha[cy.m];
+                                v = fma(cf, corner_eval<K>(jr + J::OFF_G + (2 + cy.side) * J::NG, p, cy.lam), v);
+                            }
+                            acc += v;
+                            cross = cx.state && cy.state;
+                            if (COUNT) c_corner += (cx.state != 0) + (cy.state != 0);
+                        }
+                    }
+                    const unsigned cm = __ballot_sync(0xffffffffu, cross);
+                    if (cm) {
+                        if (cross) {
+                            const int pos = nq + __popc(cm & lanemask_lt());
+                            S.qtri[pos] = tri;
+                            S.qinfo[pos] = lane | (cx.side << 5) | (cy.side << 6) | (cx.m << 7) | (cy.m << 12);
+                            S.qX[pos] = cx.X;
+                            S.qY[pos] = cy.X;
+                        }
+                        nq += __popc(cm);
+                        if (COUNT) c_cross += __popc(cm) * (lane == 0);
+                        __syncwarp();
+                        if (nq >= 32) drain<K, COUNT>(a, S, alpha, nq, lane, c_xsub);
+                    }
+                }
+            }
+        }
+    }
+    while (nq > 0) drain<K, COUNT>(a, S, alpha, nq, lane, c_xsub);
+    __syncwarp();
+    if (valid) a.out[orig] = acc + S.acc[lane];
+    if (COUNT) {
+        unsigned long long v[7] = {c_cand, c_pairs, c_pieces, c_sub, c_corner, c_cross, c_xsub};
+#pragma unroll
+        for (int i = 0; i < 7; ++i) {
+            unsigned long long x = v[i];
+            if (i >= 2 && i != 5) {
+                for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(0xffffffffu, x, o);
+            }
+            if (lane == 0 && x) atomicAdd(a.cnt + i, x);
+        }
+    }
+}
+
+}  // namespace siacjump

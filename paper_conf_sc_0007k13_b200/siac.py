@@ -23,7 +23,7 @@ LIB_PATH = os.path.join(_HERE, "libsiac_b200.so")
 if os.environ.get("SIAC_LIB_VARIANT"):
     LIB_PATH = os.path.join(_HERE, f"libsiac_b200.{os.environ['SIAC_LIB_VARIANT']}.so")
 SOURCES = [os.path.join(_HERE, "csrc", f) for f in ("siac.cu", "siac_device.cuh", "siac_tile.cuh", "siac_ws.cuh", "siac_clipfast.cuh", "siac_math.cpp",
-                                                    "siac_math.h", "siac_quadrature.h")]
+                                                    "siac_math.h", "siac_quadrature.h", "siac_jump.cuh")]
 SOURCES.append(os.path.join(os.path.dirname(_HERE), "include", "siac.h"))
 
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
@@ -60,7 +60,8 @@ class _Params(ctypes.Structure):
 
 class _Counters(ctypes.Structure):
     _fields_ = [("n_points", ctypes.c_int64), ("candidates", ctypes.c_int64), ("pairs", ctypes.c_int64),
-                ("pieces", ctypes.c_int64), ("subtris", ctypes.c_int64)]
+                ("pieces", ctypes.c_int64), ("subtris", ctypes.c_int64), ("corner_terms", ctypes.c_int64),
+                ("cross_terms", ctypes.c_int64), ("cross_subtris", ctypes.c_int64)]
 
 
 _lib = None
@@ -189,7 +190,7 @@ class Context:
         return {f: getattr(c, f) for f, _ in _Counters._fields_}
 
     def set_schedule(self, schedule: int) -> None:
-        """0 = default (fastest), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized."""
+        """0 = default (fastest = 4), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump."""
         _check(lib().siac_set_schedule(self._ptr, int(schedule)), self._ptr)
 
     def set_timing(self, on: bool = True) -> None:

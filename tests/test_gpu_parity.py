@@ -80,12 +80,44 @@ def test_cfg2_every_point(siac_mod, oracle_mod, field):
 
 
 @pytest.mark.parametrize("c", [1, 2])
-@pytest.mark.parametrize("schedule", [1, 2, 3])
+@pytest.mark.parametrize("schedule", [1, 2, 3, 4])
 def test_every_schedule_matches_oracle(siac_mod, oracle_mod, c, schedule):
-    """Every schedule (point, tile, warp-specialized) computes the same values."""
+    """Every schedule (point, tile, warp-specialized, jump) computes the same values."""
     w = cfg(c, "random")
     o = oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points)
     assert_parity(gpu_eval(siac_mod, w, schedule=schedule), o)
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 4])
+@pytest.mark.parametrize("schedule", [2, 4])
+def test_every_k_delaunay_random_field(siac_mod, oracle_mod, k, schedule):
+    """Every degree on an unstructured periodic mesh, random modes, h = max edge: the jump
+    schedule's corner polynomials and cross terms at every k against the oracle."""
+    V, T = inputs.lattice_delaunay_mesh(1500, seed=20 + k)
+    C = inputs.random_modes(len(T), k, seed=30 + k)
+    h = inputs.max_edge(V, T)
+    P = inputs.eval_points(V, T, k)[::5]
+    ctx = siac_mod.create(V, T, C, k, h)
+    ctx.set_schedule(schedule)
+    g = ctx.eval(P)
+    ctx.destroy()
+    assert_parity(g, oracle_mod.oracle_eval(V, T, C, k, h, P))
+
+
+@pytest.mark.parametrize("c,m", [(3, 400), (4, 150)])
+def test_jump_and_tile_agree_large(siac_mod, oracle_mod, c, m):
+    """cfg 3 (graded) and cfg 4 (k = 4): the jump schedule against the oracle on a sample and
+    against the clip-and-integrate schedule at every point."""
+    w = cfg(c, "random")
+    ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
+    ctx.set_schedule(4)
+    gj = ctx.eval(w.points)
+    ctx.set_schedule(2)
+    gt = ctx.eval(w.points)
+    ctx.destroy()
+    assert_parity(gj, gt)
+    idx = sample_idx(w.n_points, m, seed=100 + c)
+    assert_parity(gj[idx], oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points[idx]))
 
 
 @pytest.mark.parametrize("c,m", [(3, 1200), (4, 400), (5, 1500)])
@@ -132,12 +164,14 @@ def test_deterministic_bitwise(siac_mod):
 
 
 def test_counters_agree_between_schedules(siac_mod):
-    """Both schedules clip the same pieces: pairs, pieces and sub-triangles agree."""
+    """The clip-and-integrate schedules clip the same pieces (pairs, pieces, sub-triangles
+    agree); the jump schedule tests the same pairs and, at h = max edge, needs no general
+    clipping: one corner term per pair and axis with a knot, cross terms only where both."""
     w = cfg(2)
     ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
     ctx.set_counting(True)
     got = []
-    for sch in (0, 1, 3):
+    for sch in (2, 1, 3, 4):
         ctx.set_schedule(sch)
         ctx.eval(w.points)
         got.append(ctx.stats())
@@ -146,10 +180,16 @@ def test_counters_agree_between_schedules(siac_mod):
     assert s["n_points"] == w.n_points
     assert s["candidates"] >= s["pairs"] > 0
     assert s["subtris"] >= s["pieces"] >= s["pairs"] * 0.9
-    for o in got[1:]:
+    for o in got[1:3]:
         assert got[0]["pairs"] == o["pairs"]
         assert abs(got[0]["pieces"] - o["pieces"]) <= 1e-4 * o["pieces"]
         assert abs(got[0]["subtris"] - o["subtris"]) <= 1e-4 * o["subtris"]
+    j = got[3]
+    assert j["pairs"] == s["pairs"] and j["pieces"] == 0 and j["subtris"] == 0
+    # pieces per pair = (1 + [x knot]) (1 + [y knot]) summed, up to pieces outside the stencil
+    assert 0 < j["cross_terms"] < j["corner_terms"] < 2 * j["pairs"]
+    assert j["cross_subtris"] <= 2 * j["cross_terms"]
+    assert j["pairs"] + j["corner_terms"] + j["cross_terms"] >= s["pieces"]
 
 
 # ------------------------------------------------------------------ edge cases
