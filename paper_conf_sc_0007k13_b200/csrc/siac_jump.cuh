@@ -38,24 +38,28 @@ namespace siacjump {
 using namespace siacdev;
 
 // ------------------------------------------------------------------ jump record layout (doubles)
+// Every field group starts at an even offset so it is read with 16-byte (double2) loads.
 //   [0,1]              centroid (physical)
-//   [2..6] / [7..11]   axis x / y: zlo, zmid, zhi (sorted vertex coords, zeta frame),
-//                      invL = 1/(zmid-zlo), invR = 1/(zhi-zmid)  (0 if that corner is degenerate)
-//   [OFF_MU ..]        mu[a*(K+1)+b] = \int_T zeta1^a zeta2^b u dzeta, a, b = 0..K
-//   [OFF_G ..]         4 corners (x-right, x-left, y-top, y-bottom) x NG coefficients:
+//   [2..7] / [8..13]   axis x / y: zlo, zhi, zmid, 0, invL = 1/(zmid-zlo), invR = 1/(zhi-zmid)
+//                      (sorted vertex coordinates in the zeta frame; inv = 0 for a degenerate corner)
+//   [OFF_MU ..]        mu[a*(K+1)+b] = \int_T zeta1^a zeta2^b u dzeta, a, b = 0..K (padded to even)
+//   [OFF_G ..]         4 corners (x-right, x-left, y-top, y-bottom) x NGP coefficients:
 //                      block b (= power of the other coordinate, 0..K) holds G_b[0..K+b]
 //   [OFF_GEO ..]       per axis: L, Mv, R (vertices sorted by that coordinate), C' (the point of
 //                      edge L-R at coordinate Mv) -- 8 doubles per axis
 //   [OFF_MAP ..]       rho = m00 z1 + m01 z2 + r0, sigma = m10 z1 + m11 z2 + s0 (centred reference
 //                      coordinates of the record's modes, rho = 3r-1, sigma = 3s-1)
 //   [OFF_D ..]         modes d in centred monomials, Horner order (siac_device.cuh, Rec<K>)
+// [0, OFF_GEO) is what every (tile, candidate) step reads; the rest only the cross terms.
 template <int K> struct JRec {
     static constexpr int NB = (K + 1) * (K + 2) / 2;
     static constexpr int NG = (K + 1) * (3 * K + 2) / 2;
+    static constexpr int NGP = (NG + 1) & ~1;
+    static constexpr int NMU = (K + 1) * (K + 1);
     static constexpr int OFF_AX = 2;
-    static constexpr int OFF_MU = 12;
-    static constexpr int OFF_G = OFF_MU + (K + 1) * (K + 1);
-    static constexpr int OFF_GEO = OFF_G + 4 * NG;
+    static constexpr int OFF_MU = 14;
+    static constexpr int OFF_G = OFF_MU + ((NMU + 1) & ~1);
+    static constexpr int OFF_GEO = OFF_G + 4 * NGP;
     static constexpr int OFF_MAP = OFF_GEO + 16;
     static constexpr int OFF_D = OFF_MAP + 6;
     static constexpr int RAW = OFF_D + NB;
@@ -140,6 +144,7 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
             }
         }
         for (int i = 0; i < (K + 1) * (K + 1); ++i) o[J::OFF_MU + i] = mu[i];
+        for (int i = J::OFF_MU + J::NMU; i < J::OFF_G; ++i) o[i] = 0.0;
     }
     for (int ax = 0; ax < 2; ++ax) {
         const double *cA = ax == 0 ? zx : zy;   // coordinate along the cut axis
@@ -151,10 +156,10 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
         const double lo = cA[iL], mid = cA[iM], hi = cA[iR];
         const double f = (mid - lo) / (hi - lo);
         const double Cx = Lx + f * (Rx - Lx), Cy = Ly + f * (Ry - Ly);
-        double *ad = o + J::OFF_AX + 5 * ax;
-        ad[0] = lo; ad[1] = mid; ad[2] = hi;
-        ad[3] = mid > lo ? 1.0 / (mid - lo) : 0.0;
-        ad[4] = hi > mid ? 1.0 / (hi - mid) : 0.0;
+        double *ad = o + J::OFF_AX + 6 * ax;
+        ad[0] = lo; ad[1] = hi; ad[2] = mid; ad[3] = 0.0;
+        ad[4] = mid > lo ? 1.0 / (mid - lo) : 0.0;
+        ad[5] = hi > mid ? 1.0 / (hi - mid) : 0.0;
         double *geo = o + J::OFF_GEO + 8 * ax;
         geo[0] = Lx; geo[1] = Ly; geo[2] = Mx; geo[3] = My; geo[4] = Rx; geo[5] = Ry; geo[6] = Cx; geo[7] = Cy;
         for (int side = 0; side < 2; ++side) {      // 0: apex = R (right/top), 1: apex = L
@@ -182,8 +187,8 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
                     if (b < K) pmul_lin<2 * K + 1>(w, deg, aO, dO);
                 }
             }
-            double *go = o + J::OFF_G + (2 * ax + side) * J::NG;
-            for (int i = 0; i < J::NG; ++i) go[i] = area > 0.0 ? g[i] : 0.0;
+            double *go = o + J::OFF_G + (2 * ax + side) * J::NGP;
+            for (int i = 0; i < J::NGP; ++i) go[i] = (area > 0.0 && i < J::NG) ? g[i] : 0.0;
         }
     }
     double *mp = o + J::OFF_MAP;
@@ -191,6 +196,7 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
     for (int j = 0; j < R::NB; ++j) o[J::OFF_D + j] = dm[j];
     for (int j = J::RAW; j < J::RS; ++j) o[j] = 0.0;
 }
+
 
 // ------------------------------------------------------------------ evaluation
 
@@ -200,16 +206,25 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
 #ifndef SIAC_JUMP_MINB
 #define SIAC_JUMP_MINB 4
 #endif
+#ifndef SIAC_JUMP_PREFETCH
+#define SIAC_JUMP_PREFETCH 2      // candidates ahead whose hot record lines are prefetched into L1
+#endif
 constexpr int WARPS = SIAC_JUMP_WARPS;
 constexpr int QCAP = 64;      // cross-term queue: < 32 left over + 32 new
+constexpr int SCAP = 96;      // staged cross sub-triangles: < 32 left over + <= 64 new
 
 struct WarpSmem {
+    // cross-term queue (one entry per lane with a knot on both axes)
     int qtri[QCAP];
     int qinfo[QCAP];          // lane | sx << 5 | sy << 6 | mx << 7 | my << 12
     double qX[QCAP], qY[QCAP];
+    // staged cross sub-triangles (compacted; integrated 32 at a time)
+    double s0x[SCAP], s0y[SCAP], s1x[SCAP], s1y[SCAP], s2x[SCAP], s2y[SCAP];
+    double sX[SCAP], sY[SCAP];
+    int stri[SCAP], sinfo[SCAP];
     double acc[32];
     double4 cbox[32];
-    double px[32], py[32];
+    int klist[32];            // kept candidates of the current chunk (box meets the tile's stencils)
 };
 
 struct JumpArgs {
@@ -228,45 +243,55 @@ struct JumpArgs {
     unsigned long long *cnt;  // candidates, pairs, pieces, subtris, corner, cross, cross_subtris
 };
 
+__device__ __forceinline__ double2 ld2(const double *p) { return __ldg(reinterpret_cast<const double2 *>(p)); }
+
 struct Cut {
-    int state;     // 0 none, 1 one knot, 2 several knots (general path)
-    int base;      // base cell (may be outside 0..NC-1: zero polynomial)
+    bool cut;      // a knot lies strictly inside the triangle's range on this axis
+    bool multi;    // (GEN only) two or more knots inside: the pair takes the general path
+    int row;       // row of the base cell in the padded cell table (0 = zero polynomial)
+    int m;         // knot index (0..NC) if cut
     int side;      // 0: corner on the high side (apex = max vertex), 1: low side
-    int m;         // knot index
+    double e;      // zeta offset of the base cell: tau = zeta + e (tau = cell-centred kernel variable)
     double X;      // knot position in the zeta frame
     double lam;    // homothety ratio of the corner
 };
 
-template <int K>
+// Cut structure of one axis for a pair: dl = (centroid + image shift - x)/h on this axis.
+// GEN = false: the launcher guarantees every triangle extent is <= h (the paper's h = longest
+// edge), so two knots can only appear inside a range of length <= 1 by rounding, one of them
+// within rounding of an end; that knot's sliver is empty to rounding and is dropped.
+template <int K, bool GEN>
 __device__ __forceinline__ Cut axis_cut(const double *ad, double dl) {
     constexpr int NC = 3 * K + 1;
     constexpr double T0 = -0.5 * (3 * K + 1);
-    const double zlo = __ldg(ad + 0), zmid = __ldg(ad + 1), zhi = __ldg(ad + 2);
-    const double lo = (zlo + dl) - T0, hi = (zhi + dl) - T0;
+    const double2 lh = ld2(ad), mz = ld2(ad + 2), iv = ld2(ad + 4);
+    const double zlo = lh.x, zhi = lh.y, zmid = mz.x;
+    const double lo = (zlo + dl) - T0, hi = (zhi + dl) - T0;    // range in knot-index units
     const double fl = floor(lo);
-    const int m1 = max((int)fl + 1, 0), m2 = min((int)ceil(hi) - 1, NC);
+    double mk = fmax(fl + 1.0, 0.0);                            // first real knot above lo
     Cut c;
-    c.state = m2 < m1 ? 0 : (m2 == m1 ? 1 : 2);
-    c.m = m1;
-    c.X = (T0 + m1) - dl;
-    c.base = (int)fl;
-    c.side = 0;
-    c.lam = 0.0;
-    if (c.state == 1) {
-        if (c.X > zmid) { c.side = 0; c.base = m1 - 1; c.lam = (zhi - c.X) * __ldg(ad + 4); }
-        else { c.side = 1; c.base = m1; c.lam = (c.X - zlo) * __ldg(ad + 3); }
+    c.multi = false;
+    if (GEN) {
+        c.multi = mk + 1.0 < hi && mk + 1.0 <= (double)NC;
+    } else if (mk + 1.0 < hi && mk - lo < hi - (mk + 1.0)) {
+        mk += 1.0;                                              // rounding-only second knot
     }
+    c.cut = mk < hi && mk <= (double)NC;
+    c.X = (T0 + mk) - dl;
+    const bool hi_side = c.X > zmid;
+    c.side = hi_side ? 0 : 1;
+    const double base = c.cut ? (hi_side ? mk - 1.0 : mk) : fl;
+    c.row = (base < 0.0 || base >= (double)NC) ? 0 : (int)base + 1;
+    c.m = (int)mk;
+    c.e = dl - (T0 + base + 0.5);
+    c.lam = hi_side ? (zhi - c.X) * iv.y : (c.X - zlo) * iv.x;
     return c;
 }
 
-// Taylor coefficients p_a (a = 0..K) of P_base(zeta + dl) in powers of zeta.  kcp: padded cell
-// table, row i+1 = cell i, rows 0 and NC+1 zero.
+// Taylor coefficients p_a (a = 0..K) of the base cell polynomial at tau = zeta + e, in powers of
+// zeta.  kcp: padded cell table, row i+1 = cell i, rows 0 and NC+1 zero.
 template <int K>
-__device__ __forceinline__ void base_taylor(const double *kcp, int base, double dl, double *p) {
-    constexpr int NC = 3 * K + 1;
-    constexpr double T0 = -0.5 * (3 * K + 1);
-    const int row = (base < 0 || base >= NC) ? 0 : base + 1;
-    const double e = dl - (T0 + base + 0.5);
+__device__ __forceinline__ void base_taylor(const double *kcp, int row, double e, double *p) {
 #pragma unroll
     for (int j = 0; j <= K; ++j) p[j] = kcp[row * (K + 1) + j];
 #pragma unroll
@@ -275,22 +300,30 @@ __device__ __forceinline__ void base_taylor(const double *kcp, int base, double 
         for (int j = K - 1; j >= i; --j) p[j] = fma(e, p[j + 1], p[j]);
 }
 
-// lambda^{K+2} sum_b c_b G_b(lambda), G_b of degree K + b
+// lambda^{K+2} sum_b c_b G_b(lambda), G_b of degree K + b (corner block of NGP doubles):
+// w_j = sum_b c_b g_bj first (independent short chains), then one Horner pass in lambda.
 template <int K>
 __device__ __forceinline__ double corner_eval(const double *G, const double *c, double lam) {
-    double s = 0.0;
+    constexpr int NGP = JRec<K>::NGP;
+    double g[NGP];
 #pragma unroll
-    for (int b = K; b >= 0; --b) {
-        const double *gb = G + g_off(K, b);
-        double v = __ldg(gb + K + b);
+    for (int i = 0; i < NGP; i += 2) { const double2 v = ld2(G + i); g[i] = v.x; g[i + 1] = v.y; }
+    double w[2 * K + 1];
 #pragma unroll
-        for (int j = K + b - 1; j >= 0; --j) v = fma(v, lam, __ldg(gb + j));
-        s = fma(c[b], v, s);
+    for (int j = 0; j <= 2 * K; ++j) {
+        double t = 0.0;
+#pragma unroll
+        for (int b = K; b >= 0; --b)
+            if (j <= K + b) t = fma(c[b], g[g_off(K, b) + j], t);
+        w[j] = t;
     }
-    double l2 = lam * lam, lp = l2;
+    double v = w[2 * K];
+#pragma unroll
+    for (int j = 2 * K - 1; j >= 0; --j) v = fma(v, lam, w[j]);
+    double lp = lam * lam;
 #pragma unroll
     for (int i = 0; i < K; ++i) lp *= lam;
-    return lp * s;
+    return lp * v;
 }
 
 // \int over triangle (p0, p1, p2) of (z1 - X)^K (z2 - Y)^K u(z), rule exact for degree 3K
@@ -359,6 +392,17 @@ __device__ __forceinline__ unsigned lanemask_lt() {
     return m;
 }
 
+__device__ __forceinline__ int warp_excl_scan(int v, int lane, int &total) {
+    int s = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, s, o);
+        if (lane >= o) s += t;
+    }
+    total = __shfl_sync(0xffffffffu, s, 31);
+    return s - v;
+}
+
 // Sum v over lanes with equal key (keys >= 32 ignored), in lane order, into S.acc[key].
 __device__ __forceinline__ void seg_add(WarpSmem &S, int key, double v, int lane) {
     const unsigned grp = __match_any_sync(0xffffffffu, key);
@@ -374,68 +418,118 @@ __device__ __forceinline__ void seg_add(WarpSmem &S, int key, double v, int lane
     __syncwarp();
 }
 
-// Integrate `take` queued cross terms (from the top of the queue), one per lane.
+template <class T> __device__ __forceinline__ T pick3(int a, T v0, T v1, T v2) {
+    return a == 0 ? v0 : (a == 1 ? v1 : v2);
+}
+
+// Clip the top `take` queued cross terms (one per lane): corner_x = the homothetic corner of the
+// x knot (apex A, P1 on A-Mv, P2 on A-C'), Sutherland-Hodgman-clipped (Alg. 1) by z2 = Y on the
+// y corner's side -- a triangle, a quadrilateral (two fan triangles) or nothing; the fan
+// sub-triangles are appended, compacted, to the staging buffer.
 template <int K, bool COUNT>
-__device__ __forceinline__ void drain(const JumpArgs &a, WarpSmem &S, const double *alpha, int &nq, int lane,
-                                      unsigned long long &c_xsub) {
+__device__ __forceinline__ void clip_stage(const JumpArgs &a, WarpSmem &S, int &nq, int &ns, int lane,
+                                           unsigned long long &c_xsub) {
     using J = JRec<K>;
     const int take = min(nq, 32);
+    int nsub = 0;
+    double ax_ = 0, ay_ = 0, bx_ = 0, by_ = 0, cx_ = 0, cy_ = 0, dx_ = 0, dy_ = 0;
+    int tri = 0, info = 0;
+    double X = 0, Y = 0;
+    if (lane < take) {
+        const int e = nq - 1 - lane;
+        tri = S.qtri[e];
+        info = S.qinfo[e];
+        X = S.qX[e];
+        Y = S.qY[e];
+        const int sx = (info >> 5) & 1, sy = (info >> 6) & 1;
+        const double *jr = a.jrec + (int64_t)J::RS * tri;
+        const double2 lh = ld2(jr + J::OFF_AX), iv = ld2(jr + J::OFF_AX + 4);
+        const double lam = sx == 0 ? (lh.y - X) * iv.y : (X - lh.x) * iv.x;
+        const double *geo = jr + J::OFF_GEO;
+        const double2 A = ld2(geo + (sx == 0 ? 4 : 0)), M = ld2(geo + 2), Cp = ld2(geo + 6);
+        const double v0x = A.x, v0y = A.y;
+        const double v1x = fma(lam, M.x - A.x, A.x), v1y = fma(lam, M.y - A.y, A.y);
+        const double v2x = fma(lam, Cp.x - A.x, A.x), v2y = fma(lam, Cp.y - A.y, A.y);
+        const double sg = sy == 0 ? 1.0 : -1.0;
+        const bool k0 = sg * (v0y - Y) >= 0.0, k1 = sg * (v1y - Y) >= 0.0, k2 = sg * (v2y - Y) >= 0.0;
+        const int nk = (int)k0 + (int)k1 + (int)k2;
+        if (nk == 3) {
+            nsub = 1;
+            ax_ = v0x; ay_ = v0y; bx_ = v1x; by_ = v1y; cx_ = v2x; cy_ = v2y;
+        } else if (nk != 0) {
+            // o = the vertex alone on its side (kept if nk == 1, dropped if nk == 2)
+            const bool want = nk == 1;
+            const int o = (k0 == want) ? 0 : ((k1 == want) ? 1 : 2);
+            const int n1 = o == 2 ? 0 : o + 1, n2 = o == 0 ? 2 : o - 1;
+            const double ox = pick3(o, v0x, v1x, v2x), oy = pick3(o, v0y, v1y, v2y);
+            const double n1x = pick3(n1, v0x, v1x, v2x), n1y = pick3(n1, v0y, v1y, v2y);
+            const double n2x = pick3(n2, v0x, v1x, v2x), n2y = pick3(n2, v0y, v1y, v2y);
+            const double i1x = fma((Y - oy) / (n1y - oy), n1x - ox, ox);    // on edge o - n1
+            const double i2x = fma((Y - oy) / (n2y - oy), n2x - ox, ox);    // on edge o - n2
+            if (want) {
+                nsub = 1;
+                ax_ = ox; ay_ = oy; bx_ = i1x; by_ = Y; cx_ = i2x; cy_ = Y;
+            } else {
+                nsub = 2;        // quad n1, n2, I2, I1 -> (n1, n2, I2) + (n1, I2, I1)
+                ax_ = n1x; ay_ = n1y; bx_ = n2x; by_ = n2y; cx_ = i2x; cy_ = Y; dx_ = i1x; dy_ = Y;
+            }
+        }
+    }
+    int total;
+    const int off = ns + warp_excl_scan(nsub, lane, total);
+    if (nsub >= 1) {
+        S.s0x[off] = ax_; S.s0y[off] = ay_; S.s1x[off] = bx_; S.s1y[off] = by_; S.s2x[off] = cx_; S.s2y[off] = cy_;
+        S.sX[off] = X; S.sY[off] = Y; S.stri[off] = tri; S.sinfo[off] = info;
+    }
+    if (nsub == 2) {
+        S.s0x[off + 1] = ax_; S.s0y[off + 1] = ay_; S.s1x[off + 1] = cx_; S.s1y[off + 1] = cy_;
+        S.s2x[off + 1] = dx_; S.s2y[off + 1] = dy_;
+        S.sX[off + 1] = X; S.sY[off + 1] = Y; S.stri[off + 1] = tri; S.sinfo[off + 1] = info;
+    }
+    nq -= take;
+    ns += total;
+    if (COUNT) c_xsub += (lane == 0) ? total : 0;
+    __syncwarp();
+}
+
+// Integrate the top min(ns, 32) staged cross sub-triangles (one per lane) and add them, times
+// sgn_x alpha_mx sgn_y alpha_my, to their points' accumulators.
+template <int K>
+__device__ __forceinline__ void integrate_stage(const JumpArgs &a, WarpSmem &S, const double *alpha, int &ns,
+                                                int lane) {
+    using J = JRec<K>;
+    const int take = min(ns, 32);
     int key = 32 + lane;
     double v = 0.0;
     if (lane < take) {
-        const int e = nq - 1 - lane;
-        const int tri = S.qtri[e], info = S.qinfo[e];
-        const double X = S.qX[e], Y = S.qY[e];
+        const int e = ns - 1 - lane;
+        const int tri = S.stri[e], info = S.sinfo[e];
         key = info & 31;
         const int sx = (info >> 5) & 1, sy = (info >> 6) & 1, mx = (info >> 7) & 31, my = (info >> 12) & 31;
         const double *jr = a.jrec + (int64_t)J::RS * tri;
-        const double *ad = jr + J::OFF_AX;
-        const double lam = sx == 0 ? (__ldg(ad + 2) - X) * __ldg(ad + 4) : (X - __ldg(ad + 0)) * __ldg(ad + 3);
-        const double *geo = jr + J::OFF_GEO;
-        const double Ax = __ldg(geo + (sx == 0 ? 4 : 0)), Ay = __ldg(geo + (sx == 0 ? 5 : 1));
-        const double p1x = fma(lam, __ldg(geo + 2) - Ax, Ax), p1y = fma(lam, __ldg(geo + 3) - Ay, Ay);
-        const double p2x = fma(lam, __ldg(geo + 6) - Ax, Ax), p2y = fma(lam, __ldg(geo + 7) - Ay, Ay);
-        // Sutherland-Hodgman clip of (A, P1, P2) by z2 = Y, keeping the y-corner's side
-        const double sgn = sy == 0 ? 1.0 : -1.0;
-        const double vx[3] = {Ax, p1x, p2x}, vy[3] = {Ay, p1y, p2y};
-        double ox[4], oy[4];
-        int n = 0;
+        double mp[6], d[J::NB];
 #pragma unroll
-        for (int i = 0; i < 3; ++i) {
-            const int j = i == 2 ? 0 : i + 1;
-            const double di = sgn * (vy[i] - Y), dj = sgn * (vy[j] - Y);
-            if (di >= 0.0) { ox[n] = vx[i]; oy[n] = vy[i]; ++n; }
-            if ((di >= 0.0) != (dj >= 0.0)) {
-                const double t = (Y - vy[i]) / (vy[j] - vy[i]);
-                ox[n] = fma(t, vx[j] - vx[i], vx[i]); oy[n] = Y; ++n;
-            }
-        }
-        if (n >= 3) {
-            double mp[6], d[J::NB];
+        for (int i = 0; i < 6; i += 2) { const double2 t = ld2(jr + J::OFF_MAP + i); mp[i] = t.x; mp[i + 1] = t.y; }
 #pragma unroll
-            for (int i = 0; i < 6; ++i) mp[i] = __ldg(jr + J::OFF_MAP + i);
-#pragma unroll
-            for (int i = 0; i < J::NB; ++i) d[i] = __ldg(jr + J::OFF_D + i);
-            v = integrate_cross<K>(ox[0], oy[0], ox[1], oy[1], ox[2], oy[2], X, Y, mp, d);
-            if (n == 4) v += integrate_cross<K>(ox[0], oy[0], ox[2], oy[2], ox[3], oy[3], X, Y, mp, d);
-            if (COUNT) c_xsub += n - 2;
-            const double cxf = sx == 0 ? alpha[mx] : -alpha[mx];
-            const double cyf = sy == 0 ? alpha[my] : -alpha[my];
-            v *= cxf * cyf;
-        }
+        for (int i = 0; i < J::NB; ++i) d[i] = __ldg(jr + J::OFF_D + i);
+        v = integrate_cross<K>(S.s0x[e], S.s0y[e], S.s1x[e], S.s1y[e], S.s2x[e], S.s2y[e], S.sX[e], S.sY[e], mp, d);
+        const double cxf = sx == 0 ? alpha[mx] : -alpha[mx];
+        const double cyf = sy == 0 ? alpha[my] : -alpha[my];
+        v *= cxf * cyf;
     }
-    nq -= take;
+    ns -= take;
     __syncwarp();
     seg_add(S, key, v, lane);
 }
 
-template <int K, bool COUNT>
+template <int K, bool COUNT, bool GEN>
 __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpArgs a) {
     using J = JRec<K>;
     constexpr int NC = 3 * K + 1;
     __shared__ double kcp[(NC + 2) * (K + 1)];
     __shared__ double alpha[NC + 1];
-    __shared__ WarpSmem wsm[WARPS];
+    extern __shared__ __align__(16) unsigned char jump_dsm[];
+    WarpSmem *wsm = reinterpret_cast<WarpSmem *>(jump_dsm);
     for (int i = threadIdx.x; i < (NC + 2) * (K + 1); i += blockDim.x) {
         const int row = i / (K + 1);
         kcp[i] = (row == 0 || row == NC + 1) ? 0.0 : a.kc[i - (K + 1)];
@@ -459,8 +553,6 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
         if (a.periodic & 1) { x1 = x1 - a.Lx * floor((x1 - a.x0) / a.Lx); if (x1 >= a.x0 + a.Lx) x1 -= a.Lx; if (x1 < a.x0) x1 = a.x0; }
         if (a.periodic & 2) { x2 = x2 - a.Ly * floor((x2 - a.y0) / a.Ly); if (x2 >= a.y0 + a.Ly) x2 -= a.Ly; if (x2 < a.y0) x2 = a.y0; }
     }
-    S.px[lane] = x1;
-    S.py[lane] = x2;
     S.acc[lane] = 0.0;
     double tx0 = valid ? x1 : 1e300, tx1 = valid ? x1 : -1e300, ty0 = valid ? x2 : 1e300, ty1 = valid ? x2 : -1e300;
 #pragma unroll
@@ -479,107 +571,150 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
     __syncwarp();
 
     double acc = 0.0;
-    int nq = 0;
+    int nq = 0, ns = 0;
+    bool general = false;     // this lane met a pair with several knots on an axis
+
     unsigned long long c_cand = 0, c_pairs = 0, c_pieces = 0, c_sub = 0, c_corner = 0, c_cross = 0, c_xsub = 0;
-    for (int R = R0; R <= R1; ++R) {
-        int r = R, qy = 0;
-        if (a.periodic & 2) { r = ((R % a.ncy) + a.ncy) % a.ncy; qy = (R - r) / a.ncy; }
-        const double rsy = qy * a.Ly;
-        int C = C0;
-        while (C <= C1) {
-            int c = C, qx = 0;
-            if (a.periodic & 1) { c = ((C % a.ncx) + a.ncx) % a.ncx; qx = (C - c) / a.ncx; }
-            const int cend = (a.periodic & 1) ? min(C1, (qx + 1) * a.ncx - 1) : C1;
-            const double rsx = qx * a.Lx;
-            const int cb = c + (cend - C);
-            int t_cur = __ldg(a.cell_start + r * a.ncx + c);
-            const int t_end = __ldg(a.cell_start + r * a.ncx + cb + 1);
-            C = cend + 1;
-            for (; t_cur < t_end; t_cur += 32) {
-                const int n = min(32, t_end - t_cur);
-                bool keep = false;
-                if (lane < n) {
-                    double4 b = a.bbox[t_cur + lane];
-                    b.x += rsx; b.z += rsx; b.y += rsy; b.w += rsy;
-                    S.cbox[lane] = b;
-                    keep = (b.x < bx1 && b.z > bx0 && b.y < by1 && b.w > by0);
-                }
-                unsigned mask = __ballot_sync(0xffffffffu, keep);
-                __syncwarp();
-                while (mask) {
-                    const int j = __ffs(mask) - 1;
-                    mask &= mask - 1;
-                    const double4 b = S.cbox[j];
-                    const bool hit = valid && (b.x < sx1 && b.z > sx0 && b.y < sy1 && b.w > sy0);
-                    const unsigned hm = __ballot_sync(0xffffffffu, hit);
-                    if (COUNT) { c_cand += __popc(__ballot_sync(0xffffffffu, valid)); c_pairs += __popc(hm); }
-                    if (hm == 0) continue;
-                    const int tri = t_cur + j;
-                    const double *jr = a.jrec + (int64_t)J::RS * tri;
-                    bool cross = false;
-                    Cut cx, cy;
-                    if (hit) {
-                        const double dx = ((__ldg(jr + 0) + rsx) - x1) * a.inv_h;
-                        const double dy = ((__ldg(jr + 1) + rsy) - x2) * a.inv_h;
-                        cx = axis_cut<K>(jr + J::OFF_AX, dx);
-                        cy = axis_cut<K>(jr + J::OFF_AX + 5, dy);
-                        if (cx.state == 2 || cy.state == 2) {
-                            // general path: several knots inside a range (h < triangle size)
-                            const GenOut go = general_pair<K, COUNT>(a.rec, kcp, tri, rsx, rsy, x1, x2, a.inv_h);
-                            acc += go.v;
-                            if (COUNT) { c_pieces += go.pieces; c_sub += go.subtris; }
-                        } else {
-                            double p[K + 1], q[K + 1];
-                            base_taylor<K>(kcp, cx.base, dx, p);
-                            base_taylor<K>(kcp, cy.base, dy, q);
-                            double v = 0.0;
-#pragma unroll
-                            for (int aa = K; aa >= 0; --aa) {
-                                double s = 0.0;
-#pragma unroll
-                                for (int bb = K; bb >= 0; --bb) s = fma(q[bb], __ldg(jr + J::OFF_MU + aa * (K + 1) + bb), s);
-                                v = fma(p[aa], s, v);
-                            }
-                            if (cx.state) {
-                                const double cf = cx.side == 0 ? alpha[cx.m] : -alpha[cx.m];
-                                v = fma(cf, corner_eval<K>(jr + J::OFF_G + cx.side * J::NG, q, cx.lam), v);
-                            }
-                            if (cy.state) {
-                                const double cf = cy.side == 0 ? alpha[cy.m] : -alpha[cy.m];
-                                v = fma(cf, corner_eval<K>(jr + J::OFF_G + (2 + cy.side) * J::NG, p, cy.lam), v);
-                            }
-                            acc += v;
-                            cross = cx.state && cy.state;
-                            if (COUNT) c_corner += (cx.state != 0) + (cy.state != 0);
-                        }
+    // Warp-uniform walk over the candidate triangles of the tile: binning-cell row runs of the
+    // tile's stencil bounds (Eq. (3)-style, periodic images unwrapped), 32 boxes tested per step,
+    // then body(tri, rsx, rsy, hit) for every candidate whose box meets the tile's stencils.
+    auto candidates = [&](auto &&body) {
+        for (int R = R0; R <= R1; ++R) {
+            int r = R, qy = 0;
+            if (a.periodic & 2) { r = ((R % a.ncy) + a.ncy) % a.ncy; qy = (R - r) / a.ncy; }
+            const double rsy = qy * a.Ly;
+            int C = C0;
+            while (C <= C1) {
+                int c = C, qx = 0;
+                if (a.periodic & 1) { c = ((C % a.ncx) + a.ncx) % a.ncx; qx = (C - c) / a.ncx; }
+                const int cend = (a.periodic & 1) ? min(C1, (qx + 1) * a.ncx - 1) : C1;
+                const double rsx = qx * a.Lx;
+                const int cb = c + (cend - C);
+                int t_cur = __ldg(a.cell_start + r * a.ncx + c);
+                const int t_end = __ldg(a.cell_start + r * a.ncx + cb + 1);
+                C = cend + 1;
+                for (; t_cur < t_end; t_cur += 32) {
+                    const int n = min(32, t_end - t_cur);
+                    bool keep = false;
+                    if (lane < n) {
+                        double4 b = a.bbox[t_cur + lane];
+                        b.x += rsx; b.z += rsx; b.y += rsy; b.w += rsy;
+                        S.cbox[lane] = b;
+                        keep = (b.x < bx1 && b.z > bx0 && b.y < by1 && b.w > by0);
                     }
-                    const unsigned cm = __ballot_sync(0xffffffffu, cross);
-                    if (cm) {
-                        if (cross) {
-                            const int pos = nq + __popc(cm & lanemask_lt());
-                            S.qtri[pos] = tri;
-                            S.qinfo[pos] = lane | (cx.side << 5) | (cy.side << 6) | (cx.m << 7) | (cy.m << 12);
-                            S.qX[pos] = cx.X;
-                            S.qY[pos] = cy.X;
-                        }
-                        nq += __popc(cm);
-                        if (COUNT) c_cross += __popc(cm) * (lane == 0);
-                        __syncwarp();
-                        if (nq >= 32) drain<K, COUNT>(a, S, alpha, nq, lane, c_xsub);
+                    const unsigned mask = __ballot_sync(0xffffffffu, keep);
+                    if (keep) S.klist[__popc(mask & lanemask_lt())] = lane;
+                    const int nk = __popc(mask);
+                    __syncwarp();
+                    // software prefetch: the hot part [0, OFF_GEO) of a record spans <= HL lines
+                    constexpr int HL = (J::OFF_GEO * 8 + 127) / 128 + 1;
+                    constexpr int PD = SIAC_JUMP_PREFETCH;
+                    if (PD > 0 && lane < HL * PD && lane / HL < nk) {
+                        const double *rp = a.jrec + (int64_t)J::RS * (t_cur + S.klist[lane / HL]);
+                        asm volatile("prefetch.global.L1 [%0];" ::"l"(reinterpret_cast<const char *>(rp) + 128 * (lane % HL)));
                     }
+                    for (int i = 0; i < nk; ++i) {
+                        const int j = S.klist[i];
+                        if (PD > 0 && lane < HL && i + PD < nk) {
+                            const double *rp = a.jrec + (int64_t)J::RS * (t_cur + S.klist[i + PD]);
+                            asm volatile("prefetch.global.L1 [%0];" ::"l"(reinterpret_cast<const char *>(rp) + 128 * lane));
+                        }
+                        const double4 b = S.cbox[j];
+                        const bool hit = valid && (b.x < sx1 && b.z > sx0 && b.y < sy1 && b.w > sy0);
+                        body(t_cur + j, rsx, rsy, hit);
+                    }
+                    __syncwarp();
                 }
             }
         }
-    }
-    while (nq > 0) drain<K, COUNT>(a, S, alpha, nq, lane, c_xsub);
+    };
+
+    candidates([&](int tri, double rsx, double rsy, bool hit) {
+        const unsigned hm = __ballot_sync(0xffffffffu, hit);
+        if (COUNT) { c_cand += __popc(__ballot_sync(0xffffffffu, valid)); c_pairs += __popc(hm); }
+        if (hm == 0) return;
+        // Every lane evaluates the closed form (no divergence); only lanes whose stencil box
+        // meets the triangle's box add it (and queue its cross term): the four terms of a pair
+        // cancel to rounding only together, so a pair is taken whole or not at all.
+        const double *jr = a.jrec + (int64_t)J::RS * tri;
+        const double2 cen = ld2(jr);
+        const double dx = ((cen.x + rsx) - x1) * a.inv_h;
+        const double dy = ((cen.y + rsy) - x2) * a.inv_h;
+        const Cut cx = axis_cut<K, GEN>(jr + J::OFF_AX, dx);
+        const Cut cy = axis_cut<K, GEN>(jr + J::OFF_AX + 6, dy);
+        bool skip = false;
+        if (GEN && (cx.multi || cy.multi)) {
+            skip = true;
+            general = general || hit;     // integrated in the second pass below
+        }
+        double p[K + 1], q[K + 1];
+        base_taylor<K>(kcp, cx.row, cx.e, p);
+        base_taylor<K>(kcp, cy.row, cy.e, q);
+        double mu[J::NMU + 1];
+#pragma unroll
+        for (int i = 0; i < J::NMU; i += 2) {
+            const double2 t = ld2(jr + J::OFF_MU + i);
+            mu[i] = t.x; mu[i + 1] = t.y;
+        }
+        double v = 0.0;
+#pragma unroll
+        for (int aa = K; aa >= 0; --aa) {
+            double s = 0.0;
+#pragma unroll
+            for (int bb = K; bb >= 0; --bb) s = fma(q[bb], mu[aa * (K + 1) + bb], s);
+            v = fma(p[aa], s, v);
+        }
+        const double ax_ = cx.cut ? (cx.side == 0 ? alpha[cx.m] : -alpha[cx.m]) : 0.0;
+        const double ay_ = cy.cut ? (cy.side == 0 ? alpha[cy.m] : -alpha[cy.m]) : 0.0;
+        v = fma(ax_, corner_eval<K>(jr + J::OFF_G + cx.side * J::NGP, q, cx.lam), v);
+        v = fma(ay_, corner_eval<K>(jr + J::OFF_G + (2 + cy.side) * J::NGP, p, cy.lam), v);
+        if (hit && !skip) acc += v;
+        const bool cross = hit && !skip && cx.cut && cy.cut;
+        if (COUNT && hit && !skip) c_corner += (int)cx.cut + (int)cy.cut;
+        const unsigned cm = __ballot_sync(0xffffffffu, cross);
+        if (cm) {
+            if (cross) {
+                const int pos = nq + __popc(cm & lanemask_lt());
+                S.qtri[pos] = tri;
+                S.qinfo[pos] = lane | (cx.side << 5) | (cy.side << 6) | (cx.m << 7) | (cy.m << 12);
+                S.qX[pos] = cx.X;
+                S.qY[pos] = cy.X;
+            }
+            nq += __popc(cm);
+            if (COUNT) c_cross += __popc(cm) * (lane == 0);
+            __syncwarp();
+            if (nq >= 32) {
+                clip_stage<K, COUNT>(a, S, nq, ns, lane, c_xsub);
+                while (ns >= 32) integrate_stage<K>(a, S, alpha, ns, lane);
+            }
+        }
+    });
+    while (nq > 0) clip_stage<K, COUNT>(a, S, nq, ns, lane, c_xsub);
+    while (ns > 0) integrate_stage<K>(a, S, alpha, ns, lane);
     __syncwarp();
+    // second pass, only for tiles that met pairs with several knots on an axis (h smaller than
+    // the triangles): those pairs take the clip-and-integrate path, out of the hot loop
+    if (GEN && __any_sync(0xffffffffu, general)) {
+        candidates([&](int tri, double rsx, double rsy, bool hit) {
+            if (!hit) return;
+            const double *jr = a.jrec + (int64_t)J::RS * tri;
+            const double2 cen = ld2(jr);
+            const Cut cx = axis_cut<K, GEN>(jr + J::OFF_AX, ((cen.x + rsx) - x1) * a.inv_h);
+            const Cut cy = axis_cut<K, GEN>(jr + J::OFF_AX + 6, ((cen.y + rsy) - x2) * a.inv_h);
+            if (cx.multi || cy.multi) {
+                const GenOut go = general_pair<K, COUNT>(a.rec, kcp, tri, rsx, rsy, x1, x2, a.inv_h);
+                acc += go.v;
+                if (COUNT) { c_pieces += go.pieces; c_sub += go.subtris; }
+            }
+        });
+    }
     if (valid) a.out[orig] = acc + S.acc[lane];
     if (COUNT) {
         unsigned long long v[7] = {c_cand, c_pairs, c_pieces, c_sub, c_corner, c_cross, c_xsub};
 #pragma unroll
         for (int i = 0; i < 7; ++i) {
             unsigned long long x = v[i];
-            if (i >= 2 && i != 5) {
+            if (i == 2 || i == 3 || i == 4) {
                 for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(0xffffffffu, x, o);
             }
             if (lane == 0 && x) atomicAdd(a.cnt + i, x);

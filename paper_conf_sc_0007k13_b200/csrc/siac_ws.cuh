@@ -115,7 +115,7 @@ __device__ __forceinline__ void mbar_wait(unsigned long long *bar, int parity) {
 }
 
 // consumer-side wait (separate function so profiles attribute the two waits separately)
-__device__ __noinline__ void mbar_wait_full(unsigned long long *bar, int parity) { mbar_wait(bar, parity); }
+__device__ __noinline__ static void mbar_wait_full(unsigned long long *bar, int parity) { mbar_wait(bar, parity); }
 
 __device__ __forceinline__ unsigned lanemask_lt() {
     unsigned m;

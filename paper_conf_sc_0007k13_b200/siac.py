@@ -22,31 +22,76 @@ LIB_PATH = os.path.join(_HERE, "libsiac_b200.so")
 # experiments only: SIAC_LIB_VARIANT=name loads libsiac_b200.<name>.so (built by tools/build_variant.py)
 if os.environ.get("SIAC_LIB_VARIANT"):
     LIB_PATH = os.path.join(_HERE, f"libsiac_b200.{os.environ['SIAC_LIB_VARIANT']}.so")
-SOURCES = [os.path.join(_HERE, "csrc", f) for f in ("siac.cu", "siac_device.cuh", "siac_tile.cuh", "siac_ws.cuh", "siac_clipfast.cuh", "siac_math.cpp",
-                                                    "siac_math.h", "siac_quadrature.h", "siac_jump.cuh")]
+SOURCES = [os.path.join(_HERE, "csrc", f) for f in (
+    "siac.cu", "siac_eval_k.cu", "siac_internal.h", "siac_device.cuh", "siac_tile.cuh", "siac_ws.cuh",
+    "siac_clipfast.cuh", "siac_jump.cuh", "siac_math.cpp", "siac_math.h", "siac_quadrature.h")]
 SOURCES.append(os.path.join(os.path.dirname(_HERE), "include", "siac.h"))
 
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
-              "-Xcompiler", "-fPIC", "-shared"]
+              "-Xcompiler", "-fPIC"]
 
 SIAC_PERIODIC_X = 1
 SIAC_PERIODIC_Y = 2
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    """Compile csrc/siac.cu for sm_100a into paper_conf_sc_0007k13_b200/libsiac_b200.so."""
-    stale = force or not os.path.exists(LIB_PATH) or any(
-        os.path.getmtime(LIB_PATH) < os.path.getmtime(s) for s in SOURCES)
-    if stale:
-        nvcc = os.environ.get("NVCC", "nvcc")
-        obj = os.path.join(_HERE, "csrc", "siac_math.o")
-        subprocess.check_call(["g++", "-O2", "-std=c++17", "-fPIC", "-c", "-o", obj,
-                               os.path.join(_HERE, "csrc", "siac_math.cpp")])
-        cmd = [nvcc] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + \
-              ["-o", LIB_PATH + ".tmp", os.path.join(_HERE, "csrc", "siac.cu"), obj]
-        subprocess.check_call(cmd)
-        os.replace(LIB_PATH + ".tmp", LIB_PATH)
-    return LIB_PATH
+def build(force: bool = False, verbose: bool = False, extra_flags=(), out_path: str | None = None) -> str:
+    """Compile the CUDA library for sm_100a into paper_conf_sc_0007k13_b200/libsiac_b200.so.
+
+    Translation units: csrc/siac.cu (C ABI, create/eval orchestration, small kernels),
+    csrc/siac_eval_k.cu once per degree k = 1..4 and schedule part p = 0..3 (-DSIAC_K=k
+    -DSIAC_PART=p; the evaluation kernels), and csrc/siac_math.cpp (host exact constants, g++).
+    Objects live in csrc/build/<lib name>/ and are rebuilt only when their sources (or the
+    flags) change; the compiles run in parallel on the available cores."""
+    lib_path = out_path or LIB_PATH
+    nvcc = os.environ.get("NVCC", "nvcc")
+    tag = os.path.basename(lib_path).replace(".so", "")
+    objdir = os.path.join(_HERE, "csrc", "build", tag)
+    os.makedirs(objdir, exist_ok=True)
+    flags = NVCC_FLAGS + list(extra_flags) + (["-Xptxas", "-v"] if verbose else [])
+    cs = lambda *f: [os.path.join(_HERE, "csrc", x) for x in f]
+    common = cs("siac_internal.h", "siac_device.cuh", "siac_quadrature.h") + [SOURCES[-1]]
+    part_deps = {0: cs("siac_jump.cuh"), 1: [], 2: cs("siac_tile.cuh", "siac_clipfast.cuh"), 3: cs("siac_ws.cuh")}
+    jobs = [(["g++", "-O2", "-std=c++17", "-fPIC", "-c", "-o", os.path.join(objdir, "siac_math.o")] + cs("siac_math.cpp"),
+             os.path.join(objdir, "siac_math.o"), cs("siac_math.cpp", "siac_math.h"))]
+    jobs.append(([nvcc] + flags + ["-c", "-o", os.path.join(objdir, "siac.o")] + cs("siac.cu"),
+                 os.path.join(objdir, "siac.o"), cs("siac.cu", "siac_jump.cuh", "siac_math.h") + common))
+    for k in (1, 2, 3, 4):
+        for part in (0, 1, 2, 3):
+            o = os.path.join(objdir, f"siac_eval_k{k}_p{part}.o")
+            jobs.append(([nvcc] + flags + [f"-DSIAC_K={k}", f"-DSIAC_PART={part}", "-c", "-o", o] + cs("siac_eval_k.cu"),
+                         o, cs("siac_eval_k.cu") + common + part_deps[part]))
+    flag_file = os.path.join(objdir, "flags.txt")
+    same_flags = os.path.exists(flag_file) and open(flag_file).read() == " ".join(flags)
+
+    def stale(o, deps):
+        return force or not same_flags or not os.path.exists(o) or any(
+            os.path.getmtime(o) < os.path.getmtime(d) for d in deps)
+    todo = [(cmd, o) for cmd, o, deps in jobs if stale(o, deps)]
+    if not todo and os.path.exists(lib_path) and all(os.path.getmtime(lib_path) >= os.path.getmtime(o) for _, o, _ in jobs):
+        return lib_path
+    running, failed = [], []
+    ncpu = max(1, len(os.sched_getaffinity(0)))
+
+    def reap(p, c):
+        out, _ = p.communicate()
+        if p.returncode:
+            failed.append((c, out))
+        elif verbose and out:
+            print(out)
+    for cmd, o in todo:
+        while len(running) >= ncpu:
+            reap(*running.pop(0))
+        running.append((subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True), cmd))
+    for p, c in running:
+        reap(p, c)
+    if failed:
+        raise RuntimeError("build failed:\n" + "\n".join(" ".join(c) + "\n" + o for c, o in failed))
+    with open(flag_file, "w") as f:
+        f.write(" ".join(flags))
+    subprocess.check_call([nvcc, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", lib_path + ".tmp"]
+                          + [o for _, o, _ in jobs])
+    os.replace(lib_path + ".tmp", lib_path)
+    return lib_path
 
 
 class SiacError(RuntimeError):

@@ -14,7 +14,7 @@ from paper_conf_sc_0007k13_b200 import inputs, siac
 cfgs = [int(c) for c in sys.argv[1:]] or [2, 3, 5]
 for c in cfgs:
     w = inputs.make_config(c)
-    P = w.points if c != 5 else w.points[: 2_000_000]
+    P = w.points if (c != 5 or os.environ.get("QT_FULL")) else w.points[: 2_000_000]
     ctx = siac.create(w.V, w.T, w.C, w.k, w.h)
     d = torch.from_numpy(np.ascontiguousarray(P)).cuda()
     outs = {}
