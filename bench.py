@@ -37,6 +37,24 @@ def flops_per_subtri(k):
     return NQ[k] * 2 * (nb + 2 * k + 8)
 
 
+# Schedule JUMP (default) computes the same integral through the spline-jump decomposition
+# (DESIGN.md §8.2); its algorithmic FP64 flops per unit, counted from the operations the
+# decomposition needs (an FMA counts 2):
+#   per (point, triangle) pair: two cut tests (10 each), two Taylor shifts of the base cell
+#     polynomials (K(K+1)/2 FMA each) and the moment contraction ((K+1)^2 + (K+1) FMA);
+#   per corner term: the G contraction (NG FMA), the Horner pass in lambda (2K FMA), the
+#     lambda^(K+2) power (K+1 mul) and the accumulate (1 FMA);
+#   per cross sub-triangle: NQ quadrature points x (affine maps 8 FMA, bivariate Horner NB-1
+#     FMA, product/weight 2 FMA, t^K: K mul) + 20 set-up.
+def jump_flops(k, pairs, corners, cross_subtris):
+    nb = (k + 1) * (k + 2) // 2
+    ng = (k + 1) * (3 * k + 2) // 2
+    f_pair = 20 + 2 * (k * (k + 1) + (k + 1) * (k + 2))
+    f_corner = 2 * (ng + 2 * k + 1) + (k + 1)
+    f_xsub = NQ[k] * (2 * (nb + 9) + k) + 20
+    return pairs * f_pair + corners * f_corner + cross_subtris * f_xsub, (f_pair, f_corner, f_xsub)
+
+
 def fp64_peak_derived(sm_mhz=1965.0, sms=148):
     """148 SMs x 64 FP64 FMA lanes/clk x 2 flops x clock (B200 datasheet 37 TFLOP/s class)."""
     return sms * 64 * 2 * sm_mhz * 1e6 / 1e12
@@ -203,8 +221,29 @@ def run_siac(args):
     ctx.eval_async(d_pts, d_out, stream)
     st = ctx.stats()
     ctx.set_counting(False)
-    cands, pairs, pieces, subtris = allreduce_sum_int([st["candidates"], st["pairs"], st["pieces"], st["subtris"]])
-    flops_step = subtris * flops_per_subtri(k)           # whole job, per step
+    cands, pairs, pieces, subtris, corners, crosses, xsub = allreduce_sum_int(
+        [st["candidates"], st["pairs"], st["pieces"], st["subtris"], st["corner_terms"], st["cross_terms"],
+         st["cross_subtris"]])
+    jump = args.schedule in (0, 4)
+    if jump:
+        # JUMP: its own algorithmic flops; general-path pairs (h < triangle size only) add
+        # their clip-and-integrate sub-triangles at the direct method's rate
+        flops_step, unit_flops = jump_flops(k, pairs, corners, xsub)
+        flops_step += subtris * flops_per_subtri(k)
+    else:
+        flops_step, unit_flops = subtris * flops_per_subtri(k), (flops_per_subtri(k),)
+    direct = None
+    if jump and args.direct_count:
+        # the direct clip-and-integrate decomposition's count (schedule TILE) for context:
+        # the model flops SURVEY §8(d) defines for the same integral
+        ctx.set_schedule(2)
+        ctx.set_counting(True)
+        ctx.eval_async(d_pts, d_out, stream)
+        sd = ctx.stats()
+        ctx.set_counting(False)
+        ctx.set_schedule(args.schedule)
+        d_pieces, d_sub = allreduce_sum_int([sd["pieces"], sd["subtris"]])
+        direct = {"pieces": d_pieces, "subtris": d_sub, "model_flops_per_step": d_sub * flops_per_subtri(k)}
 
     # per-step gather of the values (NCCL all_gather_into_tensor of padded slices)
     if world > 1:
@@ -289,8 +328,10 @@ def run_siac(args):
                      "l2": ("L2 flushed (256 MB write) between timed steps" if flush else
                             "inputs larger than L2 (points %.0f MB + triangle records %.0f MB > 126 MB)"
                             % (n_local * 16 / 1e6, len(T) * rs * 8 / 1e6)),
-                     "counts": {"candidates": cands, "pairs": pairs, "pieces": pieces, "subtris": subtris},
-                     "flops_per_subtri": flops_per_subtri(k)})
+                     "counts": {"candidates": cands, "pairs": pairs, "pieces": pieces, "subtris": subtris,
+                                "corner_terms": corners, "cross_terms": crosses, "cross_subtris": xsub},
+                     "flops_per_unit": dict(zip(["pair", "corner", "cross_subtri"] if jump else ["subtri"],
+                                                unit_flops))})
         line = {"metric": "filtered quadrature points/sec (FP64)", "value": value, "unit": "points/s",
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
@@ -301,13 +342,21 @@ def run_siac(args):
                              "measured_dfma_peak": peak_meas,
                              "frac_of_measured": (achieved / peak_meas) if achieved else None,
                              "kernel_share_of_step": (kern_ms / kern_n) / ms_step if kern_n else None,
-                             "algorithmic_flops_per_step": flops_step},
+                             "algorithmic_flops_per_step": flops_step,
+                             "flop_model": ("JUMP decomposition (DESIGN.md §8.2)" if jump else
+                                            "direct SH + fan + quadrature (SURVEY §8(d))")},
                 "e2e": {"value": e2e_val, "unit": "points/s", "h2d_bytes_per_step": int(w.n_points * 16),
                         "d2h_bytes_per_step": int(w.n_points * 8)},
-                "schedule": ["default(tile)", "point", "tile", "ws"][args.schedule],
+                "schedule": ["default(jump)", "point", "tile", "ws", "jump"][args.schedule],
                 "gpu_launches": 2 * args.steps,
                 "gpu_launches_note": "per step and rank: k_point_keys + k_eval (ours) + CUB radix-sort kernels",
                 "clocks": clk}
+        if direct is not None:
+            dm = direct["model_flops_per_step"]
+            direct["model_tflops_equivalent"] = dm / world / kern_avg_s / 1e12 if kern_avg_s > 0 else None
+            direct["note"] = ("SURVEY §8(d) model flops of the direct decomposition of the same integral / this "
+                              "kernel's time: the work the jump decomposition avoids, not executed flops")
+            line["direct_method"] = direct
     if rank == 0 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(w, max(1, w.n_points // args.ref_points))
     if rank == 0:
@@ -329,8 +378,10 @@ def main():
     ap.add_argument("--ref-points", type=int, default=4000, help="oracle sample size (points)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--schedule", type=int, default=0,
-                    help="0 = default, 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized")
+                    help="0 = default (jump), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-direct-count", dest="direct_count", action="store_false",
+                    help="skip the (untimed) direct-decomposition count run")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
