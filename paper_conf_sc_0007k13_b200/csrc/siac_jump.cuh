@@ -216,8 +216,9 @@ constexpr int SCAP = 96;      // staged cross sub-triangles: < 32 left over + <=
 struct WarpSmem {
     // cross-term queue (one entry per lane with a knot on both axes)
     int qtri[QCAP];
-    int qinfo[QCAP];          // lane | sx << 5 | sy << 6 | mx << 7 | my << 12
+    int qinfo[QCAP];          // lane | sx << 5 | sy << 6 | mx << 7 | my << 12 | row_x << 17
     double qX[QCAP], qY[QCAP];
+    double qE[QCAP], qL[QCAP]; // deferred y-corner term: base-x offset e_x, y homothety ratio
     // staged cross sub-triangles (compacted; integrated 32 at a time)
     double s0x[SCAP], s0y[SCAP], s1x[SCAP], s1y[SCAP], s2x[SCAP], s2y[SCAP];
     double sX[SCAP], sY[SCAP];
@@ -427,11 +428,13 @@ template <class T> __device__ __forceinline__ T pick3(int a, T v0, T v1, T v2) {
 // y corner's side -- a triangle, a quadrilateral (two fan triangles) or nothing; the fan
 // sub-triangles are appended, compacted, to the staging buffer.
 template <int K, bool COUNT>
-__device__ __forceinline__ void clip_stage(const JumpArgs &a, WarpSmem &S, int &nq, int &ns, int lane,
-                                           unsigned long long &c_xsub) {
+__device__ __forceinline__ void clip_stage(const JumpArgs &a, WarpSmem &S, const double *kcp, const double *alpha,
+                                           int &nq, int &ns, int lane, unsigned long long &c_xsub) {
     using J = JRec<K>;
     const int take = min(nq, 32);
     int nsub = 0;
+    int ckey = 32 + lane;
+    double cval = 0.0;
     double ax_ = 0, ay_ = 0, bx_ = 0, by_ = 0, cx_ = 0, cy_ = 0, dx_ = 0, dy_ = 0;
     int tri = 0, info = 0;
     double X = 0, Y = 0;
@@ -445,6 +448,15 @@ __device__ __forceinline__ void clip_stage(const JumpArgs &a, WarpSmem &S, int &
         const double *jr = a.jrec + (int64_t)J::RS * tri;
         const double2 lh = ld2(jr + J::OFF_AX), iv = ld2(jr + J::OFF_AX + 4);
         const double lam = sx == 0 ? (lh.y - X) * iv.y : (X - lh.x) * iv.x;
+        // the pair's y-corner term, deferred from the hot loop (it evaluates one corner per lane)
+        {
+            const int my = (info >> 12) & 31, rowx = (info >> 17) & 31;
+            double pc[K + 1];
+            base_taylor<K>(kcp, rowx, S.qE[e], pc);
+            const double ay = sy == 0 ? alpha[my] : -alpha[my];
+            cval = ay * corner_eval<K>(jr + J::OFF_G + (2 + sy) * J::NGP, pc, S.qL[e]);
+            ckey = info & 31;
+        }
         const double *geo = jr + J::OFF_GEO;
         const double2 A = ld2(geo + (sx == 0 ? 4 : 0)), M = ld2(geo + 2), Cp = ld2(geo + 6);
         const double v0x = A.x, v0y = A.y;
@@ -490,6 +502,7 @@ __device__ __forceinline__ void clip_stage(const JumpArgs &a, WarpSmem &S, int &
     ns += total;
     if (COUNT) c_xsub += (lane == 0) ? total : 0;
     __syncwarp();
+    seg_add(S, ckey, cval, lane);
 }
 
 // Integrate the top min(ns, 32) staged cross sub-triangles (one per lane) and add them, times
@@ -664,10 +677,18 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
             for (int bb = K; bb >= 0; --bb) s = fma(q[bb], mu[aa * (K + 1) + bb], s);
             v = fma(p[aa], s, v);
         }
-        const double ax_ = cx.cut ? (cx.side == 0 ? alpha[cx.m] : -alpha[cx.m]) : 0.0;
-        const double ay_ = cy.cut ? (cy.side == 0 ? alpha[cy.m] : -alpha[cy.m]) : 0.0;
-        v = fma(ax_, corner_eval<K>(jr + J::OFF_G + cx.side * J::NGP, q, cx.lam), v);
-        v = fma(ay_, corner_eval<K>(jr + J::OFF_G + (2 + cy.side) * J::NGP, p, cy.lam), v);
+        // one corner per lane here: the x corner if x is cut, else the y corner; a lane with
+        // both cut defers its y corner to the cross-term queue (clip_stage)
+        const bool ux = cx.cut;
+        const bool uy = !cx.cut && cy.cut;
+        const double am = ux ? alpha[cx.m] : (uy ? alpha[cy.m] : 0.0);
+        const int sd = ux ? cx.side : 2 + cy.side;
+        const double sg = (ux ? cx.side : cy.side) == 0 ? am : -am;
+        double cc[K + 1];
+#pragma unroll
+        for (int j = 0; j <= K; ++j) cc[j] = ux ? q[j] : p[j];
+        const double lam = ux ? cx.lam : (uy ? cy.lam : 0.0);
+        v = fma(sg, corner_eval<K>(jr + J::OFF_G + sd * J::NGP, cc, lam), v);
         if (hit && !skip) acc += v;
         const bool cross = hit && !skip && cx.cut && cy.cut;
         if (COUNT && hit && !skip) c_corner += (int)cx.cut + (int)cy.cut;
@@ -676,20 +697,22 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
             if (cross) {
                 const int pos = nq + __popc(cm & lanemask_lt());
                 S.qtri[pos] = tri;
-                S.qinfo[pos] = lane | (cx.side << 5) | (cy.side << 6) | (cx.m << 7) | (cy.m << 12);
+                S.qinfo[pos] = lane | (cx.side << 5) | (cy.side << 6) | (cx.m << 7) | (cy.m << 12) | (cx.row << 17);
                 S.qX[pos] = cx.X;
                 S.qY[pos] = cy.X;
+                S.qE[pos] = cx.e;
+                S.qL[pos] = cy.lam;
             }
             nq += __popc(cm);
             if (COUNT) c_cross += __popc(cm) * (lane == 0);
             __syncwarp();
             if (nq >= 32) {
-                clip_stage<K, COUNT>(a, S, nq, ns, lane, c_xsub);
+                clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
                 while (ns >= 32) integrate_stage<K>(a, S, alpha, ns, lane);
             }
         }
     });
-    while (nq > 0) clip_stage<K, COUNT>(a, S, nq, ns, lane, c_xsub);
+    while (nq > 0) clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
     while (ns > 0) integrate_stage<K>(a, S, alpha, ns, lane);
     __syncwarp();
     // second pass, only for tiles that met pairs with several knots on an axis (h smaller than
