@@ -40,7 +40,8 @@ using namespace siacdev;
 // ------------------------------------------------------------------ jump record layout (doubles)
 // Every field group starts at an even offset so it is read with 16-byte (double2) loads.
 //   [0,1]              centroid (physical)
-//   [2..7] / [8..13]   axis x / y: zlo, zhi, zmid, 0, invL = 1/(zmid-zlo), invR = 1/(zhi-zmid)
+//   [2..7] / [8..13]   axis x / y: zlo, zhi, zmid, zc5 = (zlo+zhi)/2 + 1/2, invL = 1/(zmid-zlo),
+//                      invR = 1/(zhi-zmid)
 //                      (sorted vertex coordinates in the zeta frame; inv = 0 for a degenerate corner)
 //   [OFF_MU ..]        mu[a*(K+1)+b] = \int_T zeta1^a zeta2^b u dzeta, a, b = 0..K (padded to even)
 //   [OFF_G ..]         4 corners (x-right, x-left, y-top, y-bottom) x NGP coefficients:
@@ -157,7 +158,7 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
         const double f = (mid - lo) / (hi - lo);
         const double Cx = Lx + f * (Rx - Lx), Cy = Ly + f * (Ry - Ly);
         double *ad = o + J::OFF_AX + 6 * ax;
-        ad[0] = lo; ad[1] = hi; ad[2] = mid; ad[3] = 0.0;
+        ad[0] = lo; ad[1] = hi; ad[2] = mid; ad[3] = 0.5 * (lo + hi) + 0.5;
         ad[4] = mid > lo ? 1.0 / (mid - lo) : 0.0;
         ad[5] = hi > mid ? 1.0 / (hi - mid) : 0.0;
         double *geo = o + J::OFF_GEO + 8 * ax;
@@ -257,35 +258,48 @@ struct Cut {
     double lam;    // homothety ratio of the corner
 };
 
-// Cut structure of one axis for a pair: dl = (centroid + image shift - x)/h on this axis.
+// Cut structure of one axis for a pair; dd = (centroid + image shift - x)/h - T0 on this axis
+// (the triangle's range is (zlo + dd, zhi + dd) in knot-index units, knots at 0..NC).
 // GEN = false: the launcher guarantees every triangle extent is <= h (the paper's h = longest
-// edge), so two knots can only appear inside a range of length <= 1 by rounding, one of them
-// within rounding of an end; that knot's sliver is empty to rounding and is dropped.
+// edge), so the range holds at most one knot strictly inside; it is the integer nearest the
+// range's centre (two knots can appear inside only by rounding when an extent equals h, one
+// within rounding of each end: either choice drops a sliver that is empty to rounding).  The
+// base cell is the one below the knot when the knot is above the middle vertex (corner on the
+// high side), else the one above; with no knot inside, the cell holding the range.
 template <int K, bool GEN>
-__device__ __forceinline__ Cut axis_cut(const double *ad, double dl) {
+__device__ __forceinline__ Cut axis_cut(const double *ad, double dd) {
     constexpr int NC = 3 * K + 1;
-    constexpr double T0 = -0.5 * (3 * K + 1);
     const double2 lh = ld2(ad), mz = ld2(ad + 2), iv = ld2(ad + 4);
-    const double zlo = lh.x, zhi = lh.y, zmid = mz.x;
-    const double lo = (zlo + dl) - T0, hi = (zhi + dl) - T0;    // range in knot-index units
-    const double fl = floor(lo);
-    double mk = fmax(fl + 1.0, 0.0);                            // first real knot above lo
+    const double lo = lh.x + dd, hi = lh.y + dd;
     Cut c;
     c.multi = false;
     if (GEN) {
+        const double fl = floor(lo);
+        const double mk = fmax(fl + 1.0, 0.0);                  // first real knot above lo
         c.multi = mk + 1.0 < hi && mk + 1.0 <= (double)NC;
-    } else if (mk + 1.0 < hi && mk - lo < hi - (mk + 1.0)) {
-        mk += 1.0;                                              // rounding-only second knot
+        c.cut = mk < hi && mk <= (double)NC;
+        c.X = mk - dd;
+        const bool hi_side = c.X > mz.x;
+        c.side = hi_side ? 0 : 1;
+        const double base = c.cut ? (hi_side ? mk - 1.0 : mk) : fl;
+        c.row = (base < 0.0 || base >= (double)NC) ? 0 : (int)base + 1;
+        c.m = (int)mk;
+        c.e = (dd - 0.5) - base;
+        c.lam = hi_side ? (hi - mk) * iv.y : (mk - lo) * iv.x;
+        return c;
     }
-    c.cut = mk < hi && mk <= (double)NC;
-    c.X = (T0 + mk) - dl;
-    const bool hi_side = c.X > zmid;
-    c.side = hi_side ? 0 : 1;
-    const double base = c.cut ? (hi_side ? mk - 1.0 : mk) : fl;
-    c.row = (base < 0.0 || base >= (double)NC) ? 0 : (int)base + 1;
-    c.m = (int)mk;
-    c.e = dl - (T0 + base + 0.5);
-    c.lam = hi_side ? (zhi - c.X) * iv.y : (c.X - zlo) * iv.x;
+    const double mk = floor(mz.y + dd);                         // knot nearest the range centre
+    const int im = (int)mk;
+    c.cut = mk > lo && mk < hi && (unsigned)im <= (unsigned)NC;
+    c.X = mk - dd;
+    const bool hs = c.X > mz.x;
+    c.side = hs ? 0 : 1;
+    const bool below = c.cut ? hs : mk >= hi;                   // base cell = the one below the knot
+    const int ib = below ? im - 1 : im;
+    c.row = (unsigned)ib < (unsigned)NC ? ib + 1 : 0;
+    c.m = im;
+    c.e = (dd - 0.5) - (below ? mk - 1.0 : mk);
+    c.lam = hs ? (hi - mk) * iv.y : (mk - lo) * iv.x;
     return c;
 }
 
@@ -651,8 +665,9 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
         // cancel to rounding only together, so a pair is taken whole or not at all.
         const double *jr = a.jrec + (int64_t)J::RS * tri;
         const double2 cen = ld2(jr);
-        const double dx = ((cen.x + rsx) - x1) * a.inv_h;
-        const double dy = ((cen.y + rsy) - x2) * a.inv_h;
+        constexpr double MT0 = 0.5 * (3 * K + 1);      // -T0
+        const double dx = fma((cen.x + rsx) - x1, a.inv_h, MT0);
+        const double dy = fma((cen.y + rsy) - x2, a.inv_h, MT0);
         const Cut cx = axis_cut<K, GEN>(jr + J::OFF_AX, dx);
         const Cut cy = axis_cut<K, GEN>(jr + J::OFF_AX + 6, dy);
         bool skip = false;
@@ -722,8 +737,9 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
             if (!hit) return;
             const double *jr = a.jrec + (int64_t)J::RS * tri;
             const double2 cen = ld2(jr);
-            const Cut cx = axis_cut<K, GEN>(jr + J::OFF_AX, ((cen.x + rsx) - x1) * a.inv_h);
-            const Cut cy = axis_cut<K, GEN>(jr + J::OFF_AX + 6, ((cen.y + rsy) - x2) * a.inv_h);
+            constexpr double MT0 = 0.5 * (3 * K + 1);
+            const Cut cx = axis_cut<K, GEN>(jr + J::OFF_AX, fma((cen.x + rsx) - x1, a.inv_h, MT0));
+            const Cut cy = axis_cut<K, GEN>(jr + J::OFF_AX + 6, fma((cen.y + rsy) - x2, a.inv_h, MT0));
             if (cx.multi || cy.multi) {
                 const GenOut go = general_pair<K, COUNT>(a.rec, kcp, tri, rsx, rsy, x1, x2, a.inv_h);
                 acc += go.v;
