@@ -31,6 +31,8 @@
 // terms are queued in shared memory and integrated 32 at a time by the full warp.
 #pragma once
 
+#include <type_traits>
+
 #include "siac_device.cuh"
 
 namespace siacjump {
@@ -229,6 +231,21 @@ struct WarpSmem {
     int klist[32];            // kept candidates of the current chunk (box meets the tile's stencils)
 };
 
+#ifndef SIAC_JUMP_STAGES
+#define SIAC_JUMP_STAGES 2        // records in flight per warp (TMA ring)
+#endif
+constexpr int NST = SIAC_JUMP_STAGES;
+static_assert((NST & (NST - 1)) == 0, "SIAC_JUMP_STAGES must be a power of two");
+
+// Per-warp TMA ring: the hot part [0, OFF_GEO) of the next candidates' records, copied global ->
+// shared by cp.async.bulk while the warp works on the current one.
+template <int K> struct WarpStage {
+    alignas(16) double rec[NST][JRec<K>::OFF_GEO];
+    unsigned long long bar[NST];
+    int hj[32];               // candidates of the chunk some lane's stencil meets (chunk index)
+    unsigned hm[32];          // their lane masks
+};
+
 struct JumpArgs {
     const double *pts;
     const int *perm;
@@ -246,6 +263,33 @@ struct JumpArgs {
 };
 
 __device__ __forceinline__ double2 ld2(const double *p) { return __ldg(reinterpret_cast<const double2 *>(p)); }
+// SM = true: p points into shared memory (a TMA-staged record), else global (read-only path)
+template <bool SM> __device__ __forceinline__ double2 ldr2(const double *p) {
+    if constexpr (SM) return *reinterpret_cast<const double2 *>(p);
+    else return ld2(p);
+}
+
+// ------------------------------------------------------------------ mbarrier + bulk copy (PTX)
+__device__ __forceinline__ unsigned su32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mb_init(unsigned long long *b, int n) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(b)), "r"(n) : "memory");
+}
+// one thread: arm the barrier with the byte count and start the copy (1D TMA, 16 B granules)
+__device__ __forceinline__ void bulk_load(void *dst, const void *src, unsigned bytes, unsigned long long *b) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(b)), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(su32(dst)), "l"(src), "r"(bytes), "r"(su32(b)) : "memory");
+}
+__device__ __forceinline__ void mb_wait(unsigned long long *b, unsigned parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred P1;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+        "@!P1 bra WAIT_%=;\n"
+        "}\n" ::"r"(su32(b)), "r"(parity)
+        : "memory");
+}
 
 struct Cut {
     bool cut;      // a knot lies strictly inside the triangle's range on this axis
@@ -266,10 +310,10 @@ struct Cut {
 // within rounding of each end: either choice drops a sliver that is empty to rounding).  The
 // base cell is the one below the knot when the knot is above the middle vertex (corner on the
 // high side), else the one above; with no knot inside, the cell holding the range.
-template <int K, bool GEN>
+template <int K, bool GEN, bool SM = false>
 __device__ __forceinline__ Cut axis_cut(const double *ad, double dd) {
     constexpr int NC = 3 * K + 1;
-    const double2 lh = ld2(ad), mz = ld2(ad + 2), iv = ld2(ad + 4);
+    const double2 lh = ldr2<SM>(ad), mz = ldr2<SM>(ad + 2), iv = ldr2<SM>(ad + 4);
     const double lo = lh.x + dd, hi = lh.y + dd;
     Cut c;
     c.multi = false;
@@ -315,14 +359,28 @@ __device__ __forceinline__ void base_taylor(const double *kcp, int row, double e
         for (int j = K - 1; j >= i; --j) p[j] = fma(e, p[j + 1], p[j]);
 }
 
+// Estrin evaluation of sum_i c[i] x^i (N coefficients): dependency depth log2(N) instead of N.
+template <int N> __device__ __forceinline__ double estrin(const double *c, double x) {
+    if constexpr (N == 1) {
+        return c[0];
+    } else {
+        constexpr int M = (N + 1) / 2;
+        double d[M];
+#pragma unroll
+        for (int i = 0; i < N / 2; ++i) d[i] = fma(c[2 * i + 1], x, c[2 * i]);
+        if constexpr (N % 2 == 1) d[M - 1] = c[N - 1];
+        return estrin<M>(d, x * x);
+    }
+}
+
 // lambda^{K+2} sum_b c_b G_b(lambda), G_b of degree K + b (corner block of NGP doubles):
-// w_j = sum_b c_b g_bj first (independent short chains), then one Horner pass in lambda.
-template <int K>
+// w_j = sum_b c_b g_bj first (independent short chains), then one Estrin pass in lambda.
+template <int K, bool SM = false>
 __device__ __forceinline__ double corner_eval(const double *G, const double *c, double lam) {
     constexpr int NGP = JRec<K>::NGP;
     double g[NGP];
 #pragma unroll
-    for (int i = 0; i < NGP; i += 2) { const double2 v = ld2(G + i); g[i] = v.x; g[i + 1] = v.y; }
+    for (int i = 0; i < NGP; i += 2) { const double2 v = ldr2<SM>(G + i); g[i] = v.x; g[i + 1] = v.y; }
     double w[2 * K + 1];
 #pragma unroll
     for (int j = 0; j <= 2 * K; ++j) {
@@ -332,12 +390,15 @@ __device__ __forceinline__ double corner_eval(const double *G, const double *c, 
             if (j <= K + b) t = fma(c[b], g[g_off(K, b) + j], t);
         w[j] = t;
     }
-    double v = w[2 * K];
+    const double v = estrin<2 * K + 1>(w, lam);
+    const double l2 = lam * lam;
+    double lp = (K & 1) ? l2 * lam : l2;            // lambda^{K+2} by squaring
+    double sq = l2;
 #pragma unroll
-    for (int j = 2 * K - 1; j >= 0; --j) v = fma(v, lam, w[j]);
-    double lp = lam * lam;
-#pragma unroll
-    for (int i = 0; i < K; ++i) lp *= lam;
+    for (int r = K / 2; r > 0; r >>= 1) {
+        if (r & 1) lp *= sq;
+        sq *= sq;
+    }
     return lp * v;
 }
 
@@ -568,9 +629,18 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
     const int lane = threadIdx.x & 31;
     const int wid = threadIdx.x >> 5;
     WarpSmem &S = wsm[wid];
+    WarpStage<K> &T = reinterpret_cast<WarpStage<K> *>(wsm + WARPS)[wid];
     const int64_t p0 = ((int64_t)blockIdx.x * WARPS + wid) * 32;
     if (p0 >= a.np) return;                       // warp-uniform
+    if (lane == 0) {
+        for (int i = 0; i < NST; ++i) mb_init(&T.bar[i], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    int g = 0;                                    // records streamed so far (ring position)
+    unsigned ph = 0;                              // per-slot phase parity
     const bool valid = p0 + lane < a.np;
+    const int nvalid = __popc(__ballot_sync(0xffffffffu, valid));
     int orig = -1;
     double x1 = 0, x2 = 0;
     if (valid) {
@@ -604,8 +674,10 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
     unsigned long long c_cand = 0, c_pairs = 0, c_pieces = 0, c_sub = 0, c_corner = 0, c_cross = 0, c_xsub = 0;
     // Warp-uniform walk over the candidate triangles of the tile: binning-cell row runs of the
     // tile's stencil bounds (Eq. (3)-style, periodic images unwrapped), 32 boxes tested per step,
-    // then body(tri, rsx, rsy, hit) for every candidate whose box meets the tile's stencils.
-    auto candidates = [&](auto &&body) {
+    // then body(tri, rsx, rsy, hit, hr) for every candidate whose box meets the tile's stencils
+    // (stg = true: only those some lane's stencil meets, hr = the record's hot part in shared
+    // memory; else hr = nullptr).
+    auto candidates = [&](auto stg, auto &&body) {
         for (int R = R0; R <= R1; ++R) {
             int r = R, qy = 0;
             if (a.periodic & 2) { r = ((R % a.ncy) + a.ncy) % a.ncy; qy = (R - r) / a.ncy; }
@@ -633,22 +705,48 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
                     if (keep) S.klist[__popc(mask & lanemask_lt())] = lane;
                     const int nk = __popc(mask);
                     __syncwarp();
-                    // software prefetch: the hot part [0, OFF_GEO) of a record spans <= HL lines
-                    constexpr int HL = (J::OFF_GEO * 8 + 127) / 128 + 1;
-                    constexpr int PD = SIAC_JUMP_PREFETCH;
-                    if (PD > 0 && lane < HL * PD && lane / HL < nk) {
-                        const double *rp = a.jrec + (int64_t)J::RS * (t_cur + S.klist[lane / HL]);
-                        asm volatile("prefetch.global.L1 [%0];" ::"l"(reinterpret_cast<const char *>(rp) + 128 * (lane % HL)));
-                    }
-                    for (int i = 0; i < nk; ++i) {
-                        const int j = S.klist[i];
-                        if (PD > 0 && lane < HL && i + PD < nk) {
-                            const double *rp = a.jrec + (int64_t)J::RS * (t_cur + S.klist[i + PD]);
-                            asm volatile("prefetch.global.L1 [%0];" ::"l"(reinterpret_cast<const char *>(rp) + 128 * lane));
+                    if constexpr (decltype(stg)::value) {
+                        // exact per-lane stencil tests against the kept boxes; compact the
+                        // candidates some lane meets, then stream their records through the ring
+                        int nh = 0;
+                        for (int i = 0; i < nk; ++i) {
+                            const int j = S.klist[i];
+                            const double4 b = S.cbox[j];
+                            const bool hit = valid && (b.x < sx1 && b.z > sx0 && b.y < sy1 && b.w > sy0);
+                            const unsigned hm = __ballot_sync(0xffffffffu, hit);
+                            if (COUNT) { c_cand += nvalid; c_pairs += __popc(hm); }
+                            if (hm) {
+                                if (lane == 0) { T.hj[nh] = j; T.hm[nh] = hm; }
+                                ++nh;
+                            }
                         }
-                        const double4 b = S.cbox[j];
-                        const bool hit = valid && (b.x < sx1 && b.z > sx0 && b.y < sy1 && b.w > sy0);
-                        body(t_cur + j, rsx, rsy, hit);
+                        __syncwarp();
+                        constexpr unsigned HB = J::OFF_GEO * 8;
+                        if (lane == 0) {
+                            for (int r = 0; r < min(NST, nh); ++r) {
+                                const int sl = (g + r) & (NST - 1);
+                                bulk_load(T.rec[sl], a.jrec + (int64_t)J::RS * (t_cur + T.hj[r]), HB, &T.bar[sl]);
+                            }
+                        }
+                        for (int i = 0; i < nh; ++i) {
+                            const int sl = (g + i) & (NST - 1);
+                            mb_wait(&T.bar[sl], (ph >> sl) & 1u);
+                            ph ^= 1u << sl;
+                            body(t_cur + T.hj[i], rsx, rsy, ((T.hm[i] >> lane) & 1u) != 0, T.rec[sl]);
+                            __syncwarp();
+                            if (lane == 0 && i + NST < nh) {
+                                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                                bulk_load(T.rec[sl], a.jrec + (int64_t)J::RS * (t_cur + T.hj[i + NST]), HB, &T.bar[sl]);
+                            }
+                        }
+                        g += nh;
+                    } else {
+                        for (int i = 0; i < nk; ++i) {
+                            const int j = S.klist[i];
+                            const double4 b = S.cbox[j];
+                            const bool hit = valid && (b.x < sx1 && b.z > sx0 && b.y < sy1 && b.w > sy0);
+                            body(t_cur + j, rsx, rsy, hit, nullptr);
+                        }
                     }
                     __syncwarp();
                 }
@@ -656,20 +754,16 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
         }
     };
 
-    candidates([&](int tri, double rsx, double rsy, bool hit) {
-        const unsigned hm = __ballot_sync(0xffffffffu, hit);
-        if (COUNT) { c_cand += __popc(__ballot_sync(0xffffffffu, valid)); c_pairs += __popc(hm); }
-        if (hm == 0) return;
+    candidates(std::true_type{}, [&](int tri, double rsx, double rsy, bool hit, const double *hr) {
         // Every lane evaluates the closed form (no divergence); only lanes whose stencil box
         // meets the triangle's box add it (and queue its cross term): the four terms of a pair
         // cancel to rounding only together, so a pair is taken whole or not at all.
-        const double *jr = a.jrec + (int64_t)J::RS * tri;
-        const double2 cen = ld2(jr);
+        const double2 cen = ldr2<true>(hr);
         constexpr double MT0 = 0.5 * (3 * K + 1);      // -T0
         const double dx = fma((cen.x + rsx) - x1, a.inv_h, MT0);
         const double dy = fma((cen.y + rsy) - x2, a.inv_h, MT0);
-        const Cut cx = axis_cut<K, GEN>(jr + J::OFF_AX, dx);
-        const Cut cy = axis_cut<K, GEN>(jr + J::OFF_AX + 6, dy);
+        const Cut cx = axis_cut<K, GEN, true>(hr + J::OFF_AX, dx);
+        const Cut cy = axis_cut<K, GEN, true>(hr + J::OFF_AX + 6, dy);
         bool skip = false;
         if (GEN && (cx.multi || cy.multi)) {
             skip = true;
@@ -681,17 +775,19 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
         double mu[J::NMU + 1];
 #pragma unroll
         for (int i = 0; i < J::NMU; i += 2) {
-            const double2 t = ld2(jr + J::OFF_MU + i);
+            const double2 t = ldr2<true>(hr + J::OFF_MU + i);
             mu[i] = t.x; mu[i + 1] = t.y;
         }
-        double v = 0.0;
+        double ve = 0.0, vo = 0.0;                       // two chains (even / odd a)
 #pragma unroll
         for (int aa = K; aa >= 0; --aa) {
             double s = 0.0;
 #pragma unroll
             for (int bb = K; bb >= 0; --bb) s = fma(q[bb], mu[aa * (K + 1) + bb], s);
-            v = fma(p[aa], s, v);
+            if (aa & 1) vo = fma(p[aa], s, vo);
+            else ve = fma(p[aa], s, ve);
         }
+        double v = ve + vo;
         // one corner per lane here: the x corner if x is cut, else the y corner; a lane with
         // both cut defers its y corner to the cross-term queue (clip_stage)
         const bool ux = cx.cut;
@@ -703,7 +799,7 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
 #pragma unroll
         for (int j = 0; j <= K; ++j) cc[j] = ux ? q[j] : p[j];
         const double lam = ux ? cx.lam : (uy ? cy.lam : 0.0);
-        v = fma(sg, corner_eval<K>(jr + J::OFF_G + sd * J::NGP, cc, lam), v);
+        v = fma(sg, corner_eval<K, true>(hr + J::OFF_G + sd * J::NGP, cc, lam), v);
         if (hit && !skip) acc += v;
         const bool cross = hit && !skip && cx.cut && cy.cut;
         if (COUNT && hit && !skip) c_corner += (int)cx.cut + (int)cy.cut;
@@ -733,7 +829,7 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
     // second pass, only for tiles that met pairs with several knots on an axis (h smaller than
     // the triangles): those pairs take the clip-and-integrate path, out of the hot loop
     if (GEN && __any_sync(0xffffffffu, general)) {
-        candidates([&](int tri, double rsx, double rsy, bool hit) {
+        candidates(std::false_type{}, [&](int tri, double rsx, double rsy, bool hit, const double *) {
             if (!hit) return;
             const double *jr = a.jrec + (int64_t)J::RS * tri;
             const double2 cen = ld2(jr);
