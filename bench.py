@@ -44,15 +44,20 @@ def flops_per_subtri(k):
 #     polynomials (K(K+1)/2 FMA each) and the moment contraction ((K+1)^2 + (K+1) FMA);
 #   per corner term: the G contraction (NG FMA), the Horner pass in lambda (2K FMA), the
 #     lambda^(K+2) power (K+1 mul) and the accumulate (1 FMA);
-#   per cross sub-triangle: NQ quadrature points x (affine maps 8 FMA, bivariate Horner NB-1
-#     FMA, product/weight 2 FMA, t^K: K mul) + 20 set-up.
-def jump_flops(k, pairs, corners, cross_subtris):
+#   per cross sub-triangle (schedule 4): NQ quadrature points x (affine maps 8 FMA, bivariate
+#     Horner NB-1 FMA, product/weight 2 FMA, t^K: K mul) + 20 set-up;
+#   per interval-polynomial cross term (schedule 5, default): 2D Clenshaw over NP = (K+1)(3K+3)
+#     Chebyshev coefficients (1 FMA + 1 add each) + lambda^(2K+2) and the mapping (~2K + 12).
+def jump_flops(k, pairs, corners, cross_subtris, cross_polys=0):
     nb = (k + 1) * (k + 2) // 2
     ng = (k + 1) * (3 * k + 2) // 2
+    npoly = (k + 1) * (3 * k + 3)
     f_pair = 20 + 2 * (k * (k + 1) + (k + 1) * (k + 2))
     f_corner = 2 * (ng + 2 * k + 1) + (k + 1)
     f_xsub = NQ[k] * (2 * (nb + 9) + k) + 20
-    return pairs * f_pair + corners * f_corner + cross_subtris * f_xsub, (f_pair, f_corner, f_xsub)
+    f_xpoly = 3 * npoly + 2 * k + 12
+    return (pairs * f_pair + corners * f_corner + cross_subtris * f_xsub + cross_polys * f_xpoly,
+            (f_pair, f_corner, f_xsub, f_xpoly))
 
 
 def fp64_peak_derived(sm_mhz=1965.0, sms=148):
@@ -221,14 +226,14 @@ def run_siac(args):
     ctx.eval_async(d_pts, d_out, stream)
     st = ctx.stats()
     ctx.set_counting(False)
-    cands, pairs, pieces, subtris, corners, crosses, xsub = allreduce_sum_int(
+    cands, pairs, pieces, subtris, corners, crosses, xsub, xpoly = allreduce_sum_int(
         [st["candidates"], st["pairs"], st["pieces"], st["subtris"], st["corner_terms"], st["cross_terms"],
-         st["cross_subtris"]])
-    jump = args.schedule in (0, 4)
+         st["cross_subtris"], st["cross_polys"]])
+    jump = args.schedule in (0, 4, 5)
     if jump:
         # JUMP: its own algorithmic flops; general-path pairs (h < triangle size only) add
         # their clip-and-integrate sub-triangles at the direct method's rate
-        flops_step, unit_flops = jump_flops(k, pairs, corners, xsub)
+        flops_step, unit_flops = jump_flops(k, pairs, corners, xsub, xpoly)
         flops_step += subtris * flops_per_subtri(k)
     else:
         flops_step, unit_flops = subtris * flops_per_subtri(k), (flops_per_subtri(k),)
@@ -329,9 +334,10 @@ def run_siac(args):
                             "inputs larger than L2 (points %.0f MB + triangle records %.0f MB > 126 MB)"
                             % (n_local * 16 / 1e6, len(T) * rs * 8 / 1e6)),
                      "counts": {"candidates": cands, "pairs": pairs, "pieces": pieces, "subtris": subtris,
-                                "corner_terms": corners, "cross_terms": crosses, "cross_subtris": xsub},
-                     "flops_per_unit": dict(zip(["pair", "corner", "cross_subtri"] if jump else ["subtri"],
-                                                unit_flops))})
+                                "corner_terms": corners, "cross_terms": crosses, "cross_subtris": xsub,
+                                "cross_polys": xpoly},
+                     "flops_per_unit": dict(zip(["pair", "corner", "cross_subtri", "cross_poly"] if jump
+                                                else ["subtri"], unit_flops))})
         line = {"metric": "filtered quadrature points/sec (FP64)", "value": value, "unit": "points/s",
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
@@ -347,7 +353,7 @@ def run_siac(args):
                                             "direct SH + fan + quadrature (SURVEY §8(d))")},
                 "e2e": {"value": e2e_val, "unit": "points/s", "h2d_bytes_per_step": int(w.n_points * 16),
                         "d2h_bytes_per_step": int(w.n_points * 8)},
-                "schedule": ["default(jump)", "point", "tile", "ws", "jump"][args.schedule],
+                "schedule": ["default(jump-x)", "point", "tile", "ws", "jump", "jump-x"][args.schedule],
                 "gpu_launches": 2 * args.steps,
                 "gpu_launches_note": "per step and rank: k_point_keys + k_eval (ours) + CUB radix-sort kernels",
                 "clocks": clk}
@@ -378,7 +384,8 @@ def main():
     ap.add_argument("--ref-points", type=int, default=4000, help="oracle sample size (points)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--schedule", type=int, default=0,
-                    help="0 = default (jump), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump")
+                    help="0 = default (jump-x), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, "
+                         "4 = jump, 5 = jump with closed-form cross terms")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-direct-count", dest="direct_count", action="store_false",
                     help="skip the (untimed) direct-decomposition count run")

@@ -70,6 +70,8 @@ typedef struct {        /* geometry counts of the last evaluation (see siac_set_
     int64_t corner_terms;  /* JUMP: closed-form corner terms (one per pair and axis with a knot) */
     int64_t cross_terms;   /* JUMP: pairs with a knot on both axes (clipped corner-corner terms) */
     int64_t cross_subtris; /* JUMP: fan sub-triangles integrated for the cross terms */
+    int64_t cross_polys;   /* JUMPX: cross terms evaluated by an interval polynomial (the rest are
+                              empty or whole-corner terms) */
 } siac_counters;
 
 /*
@@ -116,7 +118,7 @@ siac_status siac_eval_async(siac_ctx *ctx, const double *d_points_xy, int64_t n_
                             double *d_values_out, void *cuda_stream);
 
 /* Evaluation schedule (same result up to rounding):
- *   SIAC_SCHEDULE_DEFAULT (0) the fastest measured schedule (currently SIAC_SCHEDULE_JUMP);
+ *   SIAC_SCHEDULE_DEFAULT (0) the fastest measured schedule (currently SIAC_SCHEDULE_JUMPX);
  *   SIAC_SCHEDULE_POINT   (1) one thread per point, clip and integrate inline (the paper's
  *                         per-point evaluation, Alg. 2, one thread per point);
  *   SIAC_SCHEDULE_TILE    (2) one warp per tile of 32 Morton-ordered points: ballot-compacted
@@ -130,12 +132,18 @@ siac_status siac_eval_async(siac_ctx *ctx, const double *d_points_xy, int64_t n_
  *                         term + closed-form corner polynomials (precomputed per triangle at
  *                         create time) + one clipped corner-corner piece integrated by quadrature
  *                         when both axes have a knot (csrc/siac_jump.cuh).  Pairs with two knots
- *                         on an axis (h < triangle size) use the clip-and-integrate path. */
+ *                         on an axis (h < triangle size) use the clip-and-integrate path;
+ *   SIAC_SCHEDULE_JUMPX   (5) JUMP with the corner-corner pieces in closed form too: the x corner
+ *                         clipped by the y knot line is the homothetic image of a fixed reference
+ *                         corner clipped by a horizontal line, whose integral is a polynomial in
+ *                         (homothety ratio, line height) on each of two height intervals, built
+ *                         per triangle at create time (Chebyshev interpolation of exact samples). */
 #define SIAC_SCHEDULE_DEFAULT 0
 #define SIAC_SCHEDULE_POINT 1
 #define SIAC_SCHEDULE_TILE 2
 #define SIAC_SCHEDULE_WS 3
 #define SIAC_SCHEDULE_JUMP 4
+#define SIAC_SCHEDULE_JUMPX 5
 siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule);
 
 /* Enable (1) / disable (0) geometry counting in later evaluations (adds atomics; off by default). */

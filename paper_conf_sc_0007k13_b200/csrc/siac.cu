@@ -44,6 +44,7 @@ struct siac_ctx {
     // device mesh
     double *d_rec = nullptr;
     double *d_jrec = nullptr;    // schedule JUMP records (siac_jump.cuh)
+    double *d_xrec = nullptr;    // closed-form cross-term polynomials (schedule JUMP-X)
     double4 *d_bbox = nullptr;
     int *d_cell_start = nullptr;
     double *d_kc = nullptr;
@@ -56,7 +57,7 @@ struct siac_ctx {
     int64_t cap_host = 0;
     double *d_hpts = nullptr, *d_hout = nullptr;
     // counters
-    int schedule = 0;            // 0 = default (= 4), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump
+    int schedule = 0;            // 0 = default (= 5), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump, 5 = jump-x
     int *d_tile_counter = nullptr;
     int num_sms = 148;
     bool counting = false;
@@ -238,7 +239,9 @@ void eval_device(siac_ctx *c, const double *d_pts, int64_t np, double *d_out, cu
     CK(cub::DeviceRadixSort::SortPairs(c->d_cub, c->cub_bytes, kb, vb, (int)np, 0, 2 * end_bit, st));
     EvalArgs a;
     a.pts = d_pts; a.perm = vb.Current(); a.np = np; a.out = d_out;
-    a.rec = c->d_rec; a.jrec = c->d_jrec; a.bbox = c->d_bbox; a.cell_start = c->d_cell_start; a.kc = c->d_kc;
+    a.rec = c->d_rec; a.jrec = c->d_jrec; a.xrec = c->d_xrec; a.bbox = c->d_bbox; a.cell_start = c->d_cell_start;
+    a.kc = c->d_kc;
+    a.xpoly = (c->schedule == 0 || c->schedule == 5) ? 1 : 0;
     a.x0 = c->dom[0]; a.y0 = c->dom[1]; a.Lx = Lx; a.Ly = Ly;
     a.h = c->h; a.inv_h = c->inv_h; a.hw = 0.5 * (3 * c->k + 1) * c->h;
     a.cw = c->cw; a.chh = c->chh; a.ex = c->ex; a.ey = c->ey;
@@ -257,14 +260,14 @@ void eval_device(siac_ctx *c, const double *d_pts, int64_t np, double *d_out, cu
         ev_stop = c->ev[c->ev_used].second;
         ++c->ev_used;
     }
-    // schedule -> part: 0 (default) and 4 = jump (p0), 1 = point (p1), 2 = tile (p2), 3 = ws (p3)
+    // schedule -> part: 0 (default) / 5 = jump-x and 4 = jump (p0), 1 = point (p1), 2 = tile (p2), 3 = ws (p3)
     static const siac_launch_fn table[4][4] = {
         {siac_launch_eval_k1_p0, siac_launch_eval_k1_p1, siac_launch_eval_k1_p2, siac_launch_eval_k1_p3},
         {siac_launch_eval_k2_p0, siac_launch_eval_k2_p1, siac_launch_eval_k2_p2, siac_launch_eval_k2_p3},
         {siac_launch_eval_k3_p0, siac_launch_eval_k3_p1, siac_launch_eval_k3_p2, siac_launch_eval_k3_p3},
         {siac_launch_eval_k4_p0, siac_launch_eval_k4_p1, siac_launch_eval_k4_p2, siac_launch_eval_k4_p3}};
     if (c->k < 1 || c->k > 4) throw Fail{SIAC_EINTERNAL, "bad k"};
-    const int part = (c->schedule == 0 || c->schedule == 4) ? 0 : c->schedule;
+    const int part = (c->schedule == 0 || c->schedule >= 4) ? 0 : c->schedule;
     const cudaError_t e = table[c->k - 1][part](a, c->counting, c->d_tile_counter, c->num_sms, st);
     CK(e);
     CK(cudaGetLastError());
@@ -291,7 +294,7 @@ void free_ctx(siac_ctx *c) {
     if (!c) return;
     cudaSetDevice(c->device);
     for (auto &e : c->ev) { cudaEventDestroy(e.first); cudaEventDestroy(e.second); }
-    void *ptrs[] = {c->d_rec, c->d_jrec, c->d_bbox, c->d_cell_start, c->d_kc, c->d_keys[0], c->d_keys[1],
+    void *ptrs[] = {c->d_rec, c->d_jrec, c->d_xrec, c->d_bbox, c->d_cell_start, c->d_kc, c->d_keys[0], c->d_keys[1],
                     c->d_idx[0], c->d_idx[1], c->d_cub, c->d_hpts, c->d_hout, c->d_cnt, c->d_tile_counter};
     for (void *p : ptrs)
         if (p) cudaFree(p);
@@ -464,6 +467,21 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
                 case 3: CK(siac_prep_jump_k3(c->d_rec, nt, p->h, c->d_jrec)); break;
                 default: CK(siac_prep_jump_k4(c->d_rec, nt, p->h, c->d_jrec)); break;
             }
+            // closed-form cross terms (interval polynomials of the reference corners)
+            int xrs = 0;
+            switch (k) {
+                case 1: xrs = siac_xrec_doubles_k1(); break;
+                case 2: xrs = siac_xrec_doubles_k2(); break;
+                case 3: xrs = siac_xrec_doubles_k3(); break;
+                default: xrs = siac_xrec_doubles_k4(); break;
+            }
+            CK(cudaMalloc(&c->d_xrec, sizeof(double) * xrs * nt));
+            switch (k) {
+                case 1: CK(siac_prep_cross_k1(c->d_jrec, nt, c->d_xrec)); break;
+                case 2: CK(siac_prep_cross_k2(c->d_jrec, nt, c->d_xrec)); break;
+                case 3: CK(siac_prep_cross_k3(c->d_jrec, nt, c->d_xrec)); break;
+                default: CK(siac_prep_cross_k4(c->d_jrec, nt, c->d_xrec)); break;
+            }
             CK(cudaGetLastError());
             CK(cudaDeviceSynchronize());
         } catch (...) {
@@ -535,12 +553,13 @@ siac_status siac_stats(siac_ctx *ctx, siac_counters *out) {
         out->corner_terms = (int64_t)h[4];
         out->cross_terms = (int64_t)h[5];
         out->cross_subtris = (int64_t)h[6];
+        out->cross_polys = (int64_t)h[7];
     });
 }
 
 siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule) {
     if (!ctx) { g_err = "NULL context"; return SIAC_EINVAL; }
-    if (schedule < 0 || schedule > 4) { ctx->err = "unknown schedule"; return SIAC_EINVAL; }
+    if (schedule < 0 || schedule > 5) { ctx->err = "unknown schedule"; return SIAC_EINVAL; }
     ctx->schedule = schedule;
     return SIAC_OK;
 }

@@ -126,7 +126,8 @@ template <int K>
 cudaError_t launch_part(const EvalArgs &a, bool count, int *, int, cudaStream_t st) {
 
     siacjump::JumpArgs j;
-    j.pts = a.pts; j.perm = a.perm; j.np = a.np; j.out = a.out; j.rec = a.rec; j.jrec = a.jrec; j.bbox = a.bbox;
+    j.pts = a.pts; j.perm = a.perm; j.np = a.np; j.out = a.out; j.rec = a.rec; j.jrec = a.jrec; j.xrec = a.xrec;
+    j.bbox = a.bbox;
     j.cell_start = a.cell_start; j.kc = a.kc; j.x0 = a.x0; j.y0 = a.y0; j.Lx = a.Lx; j.Ly = a.Ly;
     j.inv_h = a.inv_h; j.hw = a.hw; j.cw = a.cw; j.chh = a.chh; j.ex = a.ex; j.ey = a.ey;
     j.ncx = a.ncx; j.ncy = a.ncy; j.periodic = a.periodic; j.cnt = a.cnt;
@@ -135,13 +136,15 @@ cudaError_t launch_part(const EvalArgs &a, bool count, int *, int, cudaStream_t 
     const size_t smem = (sizeof(siacjump::WarpSmem) + sizeof(siacjump::WarpStage<K>)) * siacjump::WARPS;
     // GEN: some triangle is wider than h (in x or y), so a pair may see two knots on an axis
     const bool gen = std::max(a.ex, a.ey) > a.h * (1.0 + 1e-9);
-#define SIAC_LAUNCH_JUMP(C, G)                                                                                     \
+#define SIAC_LAUNCH_JUMP(C, G, XP)                                                                             \
 do {                                                                                                           \
-    CK(cudaFuncSetAttribute(siacjump::k_eval_jump<K, C, G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
-    siacjump::k_eval_jump<K, C, G><<<grid, siacjump::WARPS * 32, smem, st>>>(j);                                  \
+    CK(cudaFuncSetAttribute(siacjump::k_eval_jump<K, C, G, XP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
+    siacjump::k_eval_jump<K, C, G, XP><<<grid, siacjump::WARPS * 32, smem, st>>>(j);                          \
 } while (0)
-    if (count) { if (gen) SIAC_LAUNCH_JUMP(true, true); else SIAC_LAUNCH_JUMP(true, false); }
-    else { if (gen) SIAC_LAUNCH_JUMP(false, true); else SIAC_LAUNCH_JUMP(false, false); }
+#define SIAC_LAUNCH_JUMP2(C, G) do { if (a.xpoly) SIAC_LAUNCH_JUMP(C, G, true); else SIAC_LAUNCH_JUMP(C, G, false); } while (0)
+    if (count) { if (gen) SIAC_LAUNCH_JUMP2(true, true); else SIAC_LAUNCH_JUMP2(true, false); }
+    else { if (gen) SIAC_LAUNCH_JUMP2(false, true); else SIAC_LAUNCH_JUMP2(false, false); }
+#undef SIAC_LAUNCH_JUMP2
 #undef SIAC_LAUNCH_JUMP
     return cudaGetLastError();
 
@@ -215,4 +218,9 @@ cudaError_t SIAC_CAT(siac_prep_jump_k, SIAC_K)(const double *rec, int64_t nt, do
     siacjump::k_prep_jump<SIAC_K><<<(unsigned)((nt + 127) / 128), 128>>>(rec, nt, h, jrec);
     return cudaGetLastError();
 }
+cudaError_t SIAC_CAT(siac_prep_cross_k, SIAC_K)(const double *jrec, int64_t nt, double *xrec) {
+    siacjump::k_prep_cross<SIAC_K><<<(unsigned)((4 * nt + 127) / 128), 128>>>(jrec, nt, xrec);
+    return cudaGetLastError();
+}
+int SIAC_CAT(siac_xrec_doubles_k, SIAC_K)() { return siacjump::XRec<SIAC_K>::RS; }
 #endif

@@ -12,13 +12,15 @@ struct EvalArgs {            // arguments of every evaluation schedule
     double *out;
     const double *rec;
     const double *jrec;
+    const double *xrec;       // closed-form cross terms (schedule JUMP-X)
     const double4 *bbox;
     const int *cell_start;
     const double *kc;
     double x0, y0, Lx, Ly, h, inv_h, hw;   // hw = W/2 (physical)
     double cw, chh, ex, ey;
     int ncx, ncy, periodic;
-    unsigned long long *cnt;  // [candidates, pairs, pieces, subtris, corner, cross, cross_subtris, -]
+    int xpoly;                // jump schedule: 1 = closed-form cross terms, 0 = clipped + quadrature
+    unsigned long long *cnt;  // [candidates, pairs, pieces, subtris, corner, cross, cross_subtris, cross_polys]
 };
 
 // per (k, schedule part): p0 = jump, p1 = point, p2 = tile, p3 = warp-specialized
@@ -27,7 +29,9 @@ struct EvalArgs {            // arguments of every evaluation schedule
                                              int num_sms, cudaStream_t st);
 #define SIAC_DECL_K(k)                                                                          \
     SIAC_DECL_KP(k, 0) SIAC_DECL_KP(k, 1) SIAC_DECL_KP(k, 2) SIAC_DECL_KP(k, 3)                 \
-    cudaError_t siac_prep_jump_k##k(const double *rec, int64_t nt, double h, double *jrec);
+    cudaError_t siac_prep_jump_k##k(const double *rec, int64_t nt, double h, double *jrec);        \
+    cudaError_t siac_prep_cross_k##k(const double *jrec, int64_t nt, double *xrec);                \
+    int siac_xrec_doubles_k##k();
 SIAC_DECL_K(1)
 SIAC_DECL_K(2)
 SIAC_DECL_K(3)

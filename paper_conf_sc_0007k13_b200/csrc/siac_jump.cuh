@@ -201,6 +201,121 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
 }
 
 
+// ------------------------------------------------------------------ closed-form cross terms
+// I11 = \int_{corner_x ∩ corner_y} (z1 - X)^K (z2 - Y)^K u.  With the homothety about the apex A
+// of the x corner (ratio lambda): zeta = A + lambda (w - A), z1 - X = lambda (w1 - M1) and
+// z2 - Y = lambda (w2 - Y'), Y' = A2 + (Y - A2) / lambda, so
+//     I11 = lambda^{2K+2} F(lambda, Y'),  F = \int_{Cx ∩ H(Y')} (w1 - M1)^K (w2 - Y')^K u(A + lambda (w - A)) dw
+// over the fixed reference corner Cx = (A, M, C') clipped (Alg. 1) by the y knot line.  For the
+// half-plane above the line, F is a polynomial in (lambda, Y') of degree K x (3K + 2) on each of
+// the two intervals between the corner's vertex heights (the clipped region is a triangle with
+// vertices affine in Y'; the integrand has total degree 3K), 0 above the corner and the full-
+// corner integral below it (the corner polynomials G).  Below the line: full minus above.  The
+// interval polynomials are built at create time by Chebyshev interpolation of exact samples
+// (each sample: SH clip of Cx + the degree-3K rule) and evaluated by Clenshaw recurrences.
+template <int K> struct XRec {
+    static constexpr int NS = 3 * K + 3;          // Y' degree + 1
+    static constexpr int NL = K + 1;              // lambda degree + 1
+    static constexpr int NP = NS * NL;
+    static constexpr int XB = (6 + 2 * NP + 1) & ~1;   // per x side: v0 v1 v2 iw0 iw1 0 | 2 x NP
+    static constexpr int RS = 2 * XB;
+};
+
+// \int over triangle (p0, p1, p2) of (w1 - M1)^K (w2 - Yp)^K u(A + lam (w - A)), degree-3K rule;
+// u in centred reference coordinates through the record's affine map mp.
+template <int K>
+__device__ double corner_piece(double p0x, double p0y, double p1x, double p1y, double p2x, double p2y, double M1,
+                               double Yp, double Ax, double Ay, double lam, const double *mp, const double *d) {
+    const double e1x = p1x - p0x, e1y = p1y - p0y, e2x = p2x - p0x, e2y = p2y - p0y;
+    const double area = 0.5 * fabs(e1x * e2y - e1y * e2x);
+    double acc = 0.0;
+    for (int q = 0; q < Rule<K>::NQ; ++q) {
+        const double w1 = p0x + qr<K>(q) * e1x + qs<K>(q) * e2x;
+        const double w2 = p0y + qr<K>(q) * e1y + qs<K>(q) * e2y;
+        const double z1 = fma(lam, w1 - Ax, Ax), z2 = fma(lam, w2 - Ay, Ay);
+        const double rho = fma(mp[0], z1, fma(mp[1], z2, mp[4]));
+        const double sig = fma(mp[2], z1, fma(mp[3], z2, mp[5]));
+        double t = (w1 - M1) * (w2 - Yp), tp = 1.0;
+        for (int i = 0; i < K; ++i) tp *= t;
+        acc = fma(qw<K>(q), tp * horner2<K>(d, rho, sig), acc);
+    }
+    return area * acc;
+}
+
+// One thread per (triangle, x side, interval): Chebyshev coefficients of F above the line.
+template <int K>
+__global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec) {
+    using J = JRec<K>;
+    using X = XRec<K>;
+    const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (idx >= 4 * nt) return;
+    const int64_t t = idx >> 2;
+    const int sx = (int)(idx >> 1) & 1, iv = (int)idx & 1;
+    const double *jr = jrec + (int64_t)J::RS * t;
+    const double *geo = jr + J::OFF_GEO;            // x axis: L, M, R, C'
+    const double Ax = sx == 0 ? geo[4] : geo[0], Ay = sx == 0 ? geo[5] : geo[1];
+    const double Mx = geo[2], My = geo[3], Cx = geo[6], Cy = geo[7];
+    double mp[6], d[J::NB];
+    for (int i = 0; i < 6; ++i) mp[i] = jr[J::OFF_MAP + i];
+    for (int i = 0; i < J::NB; ++i) d[i] = jr[J::OFF_D + i];
+    double v[3] = {Ay, My, Cy};
+    if (v[0] > v[1]) { const double tt = v[0]; v[0] = v[1]; v[1] = tt; }
+    if (v[1] > v[2]) { const double tt = v[1]; v[1] = v[2]; v[2] = tt; }
+    if (v[0] > v[1]) { const double tt = v[0]; v[0] = v[1]; v[1] = tt; }
+    double *xo = xrec + (int64_t)X::RS * t + sx * X::XB;
+    if (iv == 0) {
+        xo[0] = v[0]; xo[1] = v[1]; xo[2] = v[2];
+        xo[3] = v[1] > v[0] ? 1.0 / (v[1] - v[0]) : 0.0;
+        xo[4] = v[2] > v[1] ? 1.0 / (v[2] - v[1]) : 0.0;
+        xo[5] = 0.0;
+        for (int i = 6 + 2 * X::NP; i < X::XB; ++i) xo[i] = 0.0;
+    }
+    double *co = xo + 6 + iv * X::NP;
+    const double a = v[iv], b = v[iv + 1];
+    if (!(b > a)) {
+        for (int i = 0; i < X::NP; ++i) co[i] = 0.0;
+        return;
+    }
+    double f[X::NL][X::NS];
+    for (int il = 0; il < X::NL; ++il) {
+        const double lam = 0.5 * (cospi((2.0 * il + 1.0) / (2.0 * X::NL)) + 1.0);
+        for (int is = 0; is < X::NS; ++is) {
+            const double Yp = a + 0.5 * (cospi((2.0 * is + 1.0) / (2.0 * X::NS)) + 1.0) * (b - a);
+            // Sutherland-Hodgman clip of (A, M, C') by w2 >= Yp, fan from the first vertex
+            const double px[3] = {Ax, Mx, Cx}, py[3] = {Ay, My, Cy};
+            double qx[4], qy[4];
+            int n = 0;
+            for (int e = 0; e < 3; ++e) {
+                const int e2 = e == 2 ? 0 : e + 1;
+                const bool in0 = py[e] >= Yp, in1 = py[e2] >= Yp;
+                if (in0) { qx[n] = px[e]; qy[n] = py[e]; ++n; }
+                if (in0 != in1) {
+                    const double r = (Yp - py[e]) / (py[e2] - py[e]);
+                    qx[n] = fma(r, px[e2] - px[e], px[e]); qy[n] = Yp; ++n;
+                }
+            }
+            double F = 0.0;
+            for (int j = 1; j + 1 < n; ++j)
+                F += corner_piece<K>(qx[0], qy[0], qx[j], qy[j], qx[j + 1], qy[j + 1], Mx, Yp, Ax, Ay, lam, mp, d);
+            f[il][is] = F;
+        }
+    }
+    // discrete Chebyshev transform in Y' (s) then in lambda (mu)
+    double c1[X::NL][X::NS];
+    for (int il = 0; il < X::NL; ++il)
+        for (int j = 0; j < X::NS; ++j) {
+            double acc = 0.0;
+            for (int is = 0; is < X::NS; ++is) acc += f[il][is] * cospi((double)(j * (2 * is + 1)) / (2.0 * X::NS));
+            c1[il][j] = acc * ((j == 0 ? 1.0 : 2.0) / X::NS);
+        }
+    for (int i = 0; i < X::NL; ++i)
+        for (int j = 0; j < X::NS; ++j) {
+            double acc = 0.0;
+            for (int il = 0; il < X::NL; ++il) acc += c1[il][j] * cospi((double)(i * (2 * il + 1)) / (2.0 * X::NL));
+            co[i * X::NS + j] = acc * ((i == 0 ? 1.0 : 2.0) / X::NL);
+        }
+}
+
 // ------------------------------------------------------------------ evaluation
 
 #ifndef SIAC_JUMP_WARPS
@@ -253,13 +368,14 @@ struct JumpArgs {
     double *out;
     const double *rec;        // Rec<K> (general fallback)
     const double *jrec;       // JRec<K>
+    const double *xrec;       // XRec<K> (closed-form cross terms)
     const double4 *bbox;
     const int *cell_start;
     const double *kc;
     double x0, y0, Lx, Ly, inv_h, hw;
     double cw, chh, ex, ey;
     int ncx, ncy, periodic;
-    unsigned long long *cnt;  // candidates, pairs, pieces, subtris, corner, cross, cross_subtris
+    unsigned long long *cnt;  // candidates, pairs, pieces, subtris, corner, cross, cross_subtris, cross_polys
 };
 
 __device__ __forceinline__ double2 ld2(const double *p) { return __ldg(reinterpret_cast<const double2 *>(p)); }
@@ -610,7 +726,105 @@ __device__ __forceinline__ void integrate_stage(const JumpArgs &a, WarpSmem &S, 
     seg_add(S, key, v, lane);
 }
 
-template <int K, bool COUNT, bool GEN>
+// Clenshaw evaluation of sum_{i<NL, j<NS} c[i NS + j] T_i(mu) T_j(s) (global, per-lane record)
+template <int NL, int NS>
+__device__ __forceinline__ double cheb2d(const double *c, double mu, double s) {
+    double g[NL];
+    const double s2 = 2.0 * s;
+#pragma unroll
+    for (int i = 0; i < NL; ++i) {
+        double b1 = 0.0, b2 = 0.0;
+#pragma unroll
+        for (int j = NS - 1; j >= 1; --j) {
+            const double t = fma(s2, b1, __ldg(c + i * NS + j) - b2);
+            b2 = b1;
+            b1 = t;
+        }
+        g[i] = fma(s, b1, __ldg(c + i * NS) - b2);
+    }
+    const double m2 = 2.0 * mu;
+    double b1 = 0.0, b2 = 0.0;
+#pragma unroll
+    for (int i = NL - 1; i >= 1; --i) {
+        const double t = fma(m2, b1, g[i] - b2);
+        b2 = b1;
+        b1 = t;
+    }
+    return fma(mu, b1, g[0] - b2);
+}
+
+// Closed-form cross terms of the top min(nq, 32) queue entries (one per lane), plus their
+// deferred y-corner terms, added to the owners' accumulators.
+template <int K, bool COUNT>
+__device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmem &S, const double *kcp, const double *alpha,
+                                            int &nq, int lane, unsigned long long &c_poly) {
+    using J = JRec<K>;
+    using X = XRec<K>;
+    const int take = min(nq, 32);
+    int key = 32 + lane;
+    double val = 0.0;
+    if (lane < take) {
+        const int e = nq - 1 - lane;
+        const int tri = S.qtri[e], info = S.qinfo[e];
+        const double Xk = S.qX[e], Y = S.qY[e];
+        key = info & 31;
+        const int sx = (info >> 5) & 1, sy = (info >> 6) & 1, mx = (info >> 7) & 31, my = (info >> 12) & 31;
+        const int rowx = (info >> 17) & 31;
+        const double *jr = a.jrec + (int64_t)J::RS * tri;
+        const double ay = sy == 0 ? alpha[my] : -alpha[my];
+        const double ax = sx == 0 ? alpha[mx] : -alpha[mx];
+        // deferred y-corner term of the pair
+        double pc[K + 1];
+        base_taylor<K>(kcp, rowx, S.qE[e], pc);
+        const double ycorner = ay * corner_eval<K>(jr + J::OFF_G + (2 + sy) * J::NGP, pc, S.qL[e]);
+        // the x corner's homothety ratio and the y knot in the reference corner's frame
+        const double2 lh = ld2(jr + J::OFF_AX), iv = ld2(jr + J::OFF_AX + 4);
+        const double lam = sx == 0 ? (lh.y - Xk) * iv.y : (Xk - lh.x) * iv.x;
+        const double Ay = __ldg(jr + J::OFF_GEO + (sx == 0 ? 5 : 1));
+        const double *xb = a.xrec + (int64_t)X::RS * tri + sx * X::XB;
+        const double2 v01 = ld2(xb), v2i = ld2(xb + 2), i1 = ld2(xb + 4);
+        const double Yp = fma(Y - Ay, 1.0 / lam, Ay);
+        const bool above_all = Yp >= v2i.x;      // the line is above the corner
+        const bool below_all = Yp <= v01.x;      // ... below it
+        // the full-corner integral of (z1 - X)^K (z2 - Y)^K u: corner polynomials with the
+        // coefficients of (zeta2 - Y)^K in powers of zeta2
+        const bool need_full = sy == 0 ? below_all : !below_all;
+        double full = 0.0;
+        if (need_full) {
+            double cy[K + 1];
+            double pw = 1.0;
+#pragma unroll
+            for (int b = K; b >= 0; --b) {      // C(K, b) (-Y)^{K-b}
+                double bin = 1.0;
+#pragma unroll
+                for (int r = 0; r < K - b; ++r) bin = bin * (double)(K - r) / (double)(r + 1);
+                cy[b] = bin * pw;
+                pw *= -Y;
+            }
+            full = corner_eval<K>(jr + J::OFF_G + sx * J::NGP, cy, lam);
+        }
+        double part = 0.0;               // lambda^{2K+2} F_above(lambda, Y')
+        const bool inside = !above_all && !below_all;
+        if (inside) {
+            const bool lo = Yp < v01.y;
+            const double va = lo ? v01.x : v01.y, iw = lo ? v2i.y : i1.x;
+            const double sv = fma(2.0 * (Yp - va), iw, -1.0);
+            double l2k = lam * lam;
+#pragma unroll
+            for (int i = 0; i < K; ++i) l2k *= lam * lam;
+            part = l2k * cheb2d<X::NL, X::NS>(xb + 6 + (lo ? 0 : X::NP), 2.0 * lam - 1.0, sv);
+            if (COUNT) ++c_poly;
+        }
+        const double I11 = sy == 0 ? (inside ? part : (below_all ? full : 0.0))
+                                   : (inside ? full - part : (above_all ? full : 0.0));
+        val = fma(ax * ay, I11, ycorner);
+    }
+    nq -= take;
+    __syncwarp();
+    seg_add(S, key, val, lane);
+}
+
+template <int K, bool COUNT, bool GEN, bool XP>
 __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpArgs a) {
     using J = JRec<K>;
     constexpr int NC = 3 * K + 1;
@@ -671,7 +885,8 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
     int nq = 0, ns = 0;
     bool general = false;     // this lane met a pair with several knots on an axis
 
-    unsigned long long c_cand = 0, c_pairs = 0, c_pieces = 0, c_sub = 0, c_corner = 0, c_cross = 0, c_xsub = 0;
+    unsigned long long c_cand = 0, c_pairs = 0, c_pieces = 0, c_sub = 0, c_corner = 0, c_cross = 0, c_xsub = 0,
+                       c_xpoly = 0;
     // Warp-uniform walk over the candidate triangles of the tile: binning-cell row runs of the
     // tile's stencil bounds (Eq. (3)-style, periodic images unwrapped), 32 boxes tested per step,
     // then body(tri, rsx, rsy, hit, hr) for every candidate whose box meets the tile's stencils
@@ -818,12 +1033,20 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
             if (COUNT) c_cross += __popc(cm) * (lane == 0);
             __syncwarp();
             if (nq >= 32) {
-                clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
-                while (ns >= 32) integrate_stage<K>(a, S, alpha, ns, lane);
+                if (XP) {
+                    cross_stage<K, COUNT>(a, S, kcp, alpha, nq, lane, c_xpoly);
+                } else {
+                    clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
+                    while (ns >= 32) integrate_stage<K>(a, S, alpha, ns, lane);
+                }
             }
         }
     });
-    while (nq > 0) clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
+    if (XP) {
+        while (nq > 0) cross_stage<K, COUNT>(a, S, kcp, alpha, nq, lane, c_xpoly);
+    } else {
+        while (nq > 0) clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
+    }
     while (ns > 0) integrate_stage<K>(a, S, alpha, ns, lane);
     __syncwarp();
     // second pass, only for tiles that met pairs with several knots on an axis (h smaller than
@@ -845,11 +1068,11 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
     }
     if (valid) a.out[orig] = acc + S.acc[lane];
     if (COUNT) {
-        unsigned long long v[7] = {c_cand, c_pairs, c_pieces, c_sub, c_corner, c_cross, c_xsub};
+        unsigned long long v[8] = {c_cand, c_pairs, c_pieces, c_sub, c_corner, c_cross, c_xsub, c_xpoly};
 #pragma unroll
-        for (int i = 0; i < 7; ++i) {
+        for (int i = 0; i < 8; ++i) {
             unsigned long long x = v[i];
-            if (i == 2 || i == 3 || i == 4) {
+            if (i == 2 || i == 3 || i == 4 || i == 7) {
                 for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(0xffffffffu, x, o);
             }
             if (lane == 0 && x) atomicAdd(a.cnt + i, x);

@@ -106,7 +106,7 @@ class _Params(ctypes.Structure):
 class _Counters(ctypes.Structure):
     _fields_ = [("n_points", ctypes.c_int64), ("candidates", ctypes.c_int64), ("pairs", ctypes.c_int64),
                 ("pieces", ctypes.c_int64), ("subtris", ctypes.c_int64), ("corner_terms", ctypes.c_int64),
-                ("cross_terms", ctypes.c_int64), ("cross_subtris", ctypes.c_int64)]
+                ("cross_terms", ctypes.c_int64), ("cross_subtris", ctypes.c_int64), ("cross_polys", ctypes.c_int64)]
 
 
 _lib = None
@@ -235,7 +235,8 @@ class Context:
         return {f: getattr(c, f) for f, _ in _Counters._fields_}
 
     def set_schedule(self, schedule: int) -> None:
-        """0 = default (fastest = 4), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump."""
+        """0 = default (fastest = 5), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump,
+        5 = jump with closed-form cross terms."""
         _check(lib().siac_set_schedule(self._ptr, int(schedule)), self._ptr)
 
     def set_timing(self, on: bool = True) -> None:

@@ -80,7 +80,7 @@ def test_cfg2_every_point(siac_mod, oracle_mod, field):
 
 
 @pytest.mark.parametrize("c", [1, 2])
-@pytest.mark.parametrize("schedule", [1, 2, 3, 4])
+@pytest.mark.parametrize("schedule", [1, 2, 3, 4, 5])
 def test_every_schedule_matches_oracle(siac_mod, oracle_mod, c, schedule):
     """Every schedule (point, tile, warp-specialized, jump) computes the same values."""
     w = cfg(c, "random")
@@ -89,7 +89,7 @@ def test_every_schedule_matches_oracle(siac_mod, oracle_mod, c, schedule):
 
 
 @pytest.mark.parametrize("k", [1, 2, 3, 4])
-@pytest.mark.parametrize("schedule", [2, 4])
+@pytest.mark.parametrize("schedule", [2, 4, 5])
 def test_every_k_delaunay_random_field(siac_mod, oracle_mod, k, schedule):
     """Every degree on an unstructured periodic mesh, random modes, h = max edge: the jump
     schedule's corner polynomials and cross terms at every k against the oracle."""
@@ -104,13 +104,14 @@ def test_every_k_delaunay_random_field(siac_mod, oracle_mod, k, schedule):
     assert_parity(g, oracle_mod.oracle_eval(V, T, C, k, h, P))
 
 
+@pytest.mark.parametrize("sch", [4, 5])
 @pytest.mark.parametrize("c,m", [(3, 400), (4, 150)])
-def test_jump_and_tile_agree_large(siac_mod, oracle_mod, c, m):
-    """cfg 3 (graded) and cfg 4 (k = 4): the jump schedule against the oracle on a sample and
+def test_jump_and_tile_agree_large(siac_mod, oracle_mod, c, m, sch):
+    """cfg 3 (graded) and cfg 4 (k = 4): the jump schedules against the oracle on a sample and
     against the clip-and-integrate schedule at every point."""
     w = cfg(c, "random")
     ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
-    ctx.set_schedule(4)
+    ctx.set_schedule(sch)
     gj = ctx.eval(w.points)
     ctx.set_schedule(2)
     gt = ctx.eval(w.points)
@@ -171,7 +172,7 @@ def test_counters_agree_between_schedules(siac_mod):
     ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
     ctx.set_counting(True)
     got = []
-    for sch in (2, 1, 3, 4):
+    for sch in (2, 1, 3, 4, 5):
         ctx.set_schedule(sch)
         ctx.eval(w.points)
         got.append(ctx.stats())
@@ -190,6 +191,10 @@ def test_counters_agree_between_schedules(siac_mod):
     assert 0 < j["cross_terms"] < j["corner_terms"] < 2 * j["pairs"]
     assert j["cross_subtris"] <= 2 * j["cross_terms"]
     assert j["pairs"] + j["corner_terms"] + j["cross_terms"] >= s["pieces"]
+    x = got[4]      # closed-form cross terms: same pairs / corners / cross terms, no sub-triangles
+    assert (x["pairs"], x["corner_terms"], x["cross_terms"]) == (j["pairs"], j["corner_terms"], j["cross_terms"])
+    assert x["pieces"] == 0 and x["subtris"] == 0 and x["cross_subtris"] == 0
+    assert 0 < x["cross_polys"] <= x["cross_terms"]
 
 
 # ------------------------------------------------------------------ edge cases
