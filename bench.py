@@ -327,6 +327,12 @@ def run_siac(args):
         # whole-job algorithmic flops per launch-set / slowest rank's kernel time / ranks
         achieved = flops_step / world / kern_avg_s / 1e12 if kern_avg_s > 0 else None
         peak = fp64_peak_derived()
+        # DRAM traffic per launch: bytes/point of the committed ncu --set full capture of this
+        # kernel (profiles/r01_ncu_traffic_jumpx.json, a 2M-point subset) x this launch's points
+        traffic = None
+        tpath = os.path.join(ROOT, "profiles", "r01_ncu_traffic_jumpx.json")
+        if args.schedule in (0, 5) and os.path.exists(tpath):
+            traffic = json.load(open(tpath))["bytes_per_point"] * n_local
         cfgd = workload_desc(w, args.config)
         cfgd.update({"parallelism": f"spatial point tiles x{world} + halo, NCCL all_gather" if world > 1
                      else "single GPU",
@@ -343,7 +349,9 @@ def run_siac(args):
                 "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic", "config": cfgd,
                 "roofline": {"bound": "alu", "kernel": "k_eval", "achieved": achieved, "peak": peak,
-                             "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None, "traffic": None,
+                             "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+                             "traffic_note": "dram read+write bytes per launch, scaled from the committed ncu capture "
+                                             "(profiles/r01_ncu_traffic_jumpx.json); algorithmic ~41 B/point",
                              "peak_note": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1965 MHz (DESIGN.md)",
                              "measured_dfma_peak": peak_meas,
                              "frac_of_measured": (achieved / peak_meas) if achieved else None,

@@ -149,6 +149,40 @@ siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule);
 /* Enable (1) / disable (0) geometry counting in later evaluations (adds atomics; off by default). */
 siac_status siac_set_counting(siac_ctx *ctx, int32_t enable);
 
+/* ---- Steps either side of the path ("grid points ... used at the end of
+ * the simulation for such things as error calculations").  They need no
+ * context; device pointers are stream-ordered on `cuda_stream` (NULL = legacy default stream)
+ * and must stay valid until the stream passes the call.  Errors: SIAC_EINVAL for bad sizes or
+ * NULL pointers, SIAC_ECUDA for launch failures; message via siac_last_error(NULL). */
+
+/* Host: the collapsed Gauss-Legendre rule with n_quad^2 nodes (n_quad in 1..64) used by
+ * siac_project_async, exact to total degree 2 n_quad - 2.
+ *   rs_out  host, n_quad^2 x 2 doubles: node (r, s) on the unit triangle (point = v0 +
+ *           r (v1 - v0) + s (v2 - v0)); node q = i * n_quad + j.
+ *   w_out   host, n_quad^2 doubles: weights on the reference triangle (area 2; sum = 2). */
+siac_status siac_projection_rule(int32_t n_quad, double *rs_out, double *w_out);
+
+/* Device: points_out[(t * n_nodes + q)] = v0 + r_q (v1 - v0) + s_q (v2 - v0) of triangle t.
+ *   d_vertices_xy  n_vertices x 2;  d_triangles  n_triangles x 3 (0-based, unchecked here);
+ *   d_rs           n_nodes x 2 reference nodes;  d_points_out  n_triangles * n_nodes x 2. */
+siac_status siac_map_points_async(const double *d_vertices_xy, const int32_t *d_triangles, int64_t n_triangles,
+                                  const double *d_rs, int32_t n_nodes, double *d_points_out, void *cuda_stream);
+
+/* Device: L2 projection onto P_k (orthonormal Dubiner, SIAC_BASIS_DUBINER_ORTHONORMAL, the
+ * layout siac_create reads) of a field sampled at the siac_projection_rule nodes:
+ *   d_f             n_triangles x n_quad^2 values, element-major (node order of the rule);
+ *   d_coeffs_out    n_triangles x (k+1)(k+2)/2 modes.
+ * c_i = sum_q w_q phi_i(node_q) f_q (the element mass matrix on the reference triangle is the
+ * identity for this basis).  Exact for f in P_{2 n_quad - 2 - k}; k in 1..4, n_quad in k+1..32. */
+siac_status siac_project_async(int32_t k, int32_t n_quad, const double *d_f, int64_t n_triangles,
+                               double *d_coeffs_out, void *cuda_stream);
+
+/* Device: error norms of e = u - ref over n values, deterministic (fixed reduction order):
+ *   d_weights  n weights (e.g. quadrature weight x element area) or NULL (all 1);
+ *   d_out      3 doubles: sqrt(sum w e^2), max |e|, sum w. */
+siac_status siac_error_norms_async(const double *d_u, const double *d_ref, const double *d_weights, int64_t n,
+                                   double *d_out, void *cuda_stream);
+
 /* Counters of the last evaluation run with counting enabled (synchronises the device). */
 siac_status siac_stats(siac_ctx *ctx, siac_counters *out);
 

@@ -71,6 +71,7 @@ struct siac_ctx {
 };
 
 static thread_local std::string g_err;
+void siac_set_thread_error(const std::string &msg) { g_err = msg; }   // siac_io.cu (siac_internal.h)
 
 namespace {
 

@@ -4,6 +4,10 @@
 
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <string>
+
+// message returned by siac_last_error(NULL) on this thread (defined in siac.cu)
+void siac_set_thread_error(const std::string &msg);
 
 struct EvalArgs {            // arguments of every evaluation schedule
     const double *pts;        // input order, np x 2

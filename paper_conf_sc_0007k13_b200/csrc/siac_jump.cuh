@@ -212,11 +212,13 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
 // vertices affine in Y'; the integrand has total degree 3K), 0 above the corner and the full-
 // corner integral below it (the corner polynomials G).  Below the line: full minus above.  The
 // interval polynomials are built at create time by Chebyshev interpolation of exact samples
-// (each sample: SH clip of Cx + the degree-3K rule) and evaluated by Clenshaw recurrences.
+// (each sample: SH clip of Cx + the degree-3K rule), stored as monomials in (mu, s) on
+// [-1, 1]^2 and evaluated column-wise in mu (independent short chains) then by Estrin in s.
 template <int K> struct XRec {
     static constexpr int NS = 3 * K + 3;          // Y' degree + 1
     static constexpr int NL = K + 1;              // lambda degree + 1
-    static constexpr int NP = NS * NL;
+    static constexpr int NLP = (NL + 1) & ~1;     // padded for 16-byte loads
+    static constexpr int NP = NS * NLP;           // monomial coefficients m[j * NLP + i]: s^j mu^i
     static constexpr int XB = (6 + 2 * NP + 1) & ~1;   // per x side: v0 v1 v2 iw0 iw1 0 | 2 x NP
     static constexpr int RS = 2 * XB;
 };
@@ -308,11 +310,28 @@ __global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec) {
             for (int is = 0; is < X::NS; ++is) acc += f[il][is] * cospi((double)(j * (2 * is + 1)) / (2.0 * X::NS));
             c1[il][j] = acc * ((j == 0 ? 1.0 : 2.0) / X::NS);
         }
+    double c2[X::NL][X::NS];
     for (int i = 0; i < X::NL; ++i)
         for (int j = 0; j < X::NS; ++j) {
             double acc = 0.0;
             for (int il = 0; il < X::NL; ++il) acc += c1[il][j] * cospi((double)(i * (2 * il + 1)) / (2.0 * X::NL));
-            co[i * X::NS + j] = acc * ((i == 0 ? 1.0 : 2.0) / X::NL);
+            c2[i][j] = acc * ((i == 0 ? 1.0 : 2.0) / X::NL);
+        }
+    // Chebyshev -> monomial in both variables (T_j coefficients by the integer recurrence)
+    double tc[X::NS][X::NS];
+    for (int j = 0; j < X::NS; ++j)
+        for (int k = 0; k < X::NS; ++k) tc[j][k] = 0.0;
+    tc[0][0] = 1.0;
+    if (X::NS > 1) tc[1][1] = 1.0;
+    for (int j = 2; j < X::NS; ++j)
+        for (int k = 0; k < X::NS; ++k) tc[j][k] = (k > 0 ? 2.0 * tc[j - 1][k - 1] : 0.0) - tc[j - 2][k];
+    for (int jm = 0; jm < X::NS; ++jm)
+        for (int im = 0; im < X::NLP; ++im) {
+            double acc = 0.0;
+            if (im < X::NL)
+                for (int i = im; i < X::NL; ++i)
+                    for (int j = jm; j < X::NS; ++j) acc += tc[i][im] * tc[j][jm] * c2[i][j];
+            co[jm * X::NLP + im] = acc;
         }
 }
 
@@ -726,31 +745,21 @@ __device__ __forceinline__ void integrate_stage(const JumpArgs &a, WarpSmem &S, 
     seg_add(S, key, v, lane);
 }
 
-// Clenshaw evaluation of sum_{i<NL, j<NS} c[i NS + j] T_i(mu) T_j(s) (global, per-lane record)
-template <int NL, int NS>
-__device__ __forceinline__ double cheb2d(const double *c, double mu, double s) {
-    double g[NL];
-    const double s2 = 2.0 * s;
+// sum_{j<NS, i<NL} m[j NLP + i] mu^i s^j: NS independent Horner chains in mu, then Estrin in s
+template <int NL, int NLP, int NS>
+__device__ __forceinline__ double mono2d(const double *m, double mu, double s) {
+    double col[NS];
 #pragma unroll
-    for (int i = 0; i < NL; ++i) {
-        double b1 = 0.0, b2 = 0.0;
+    for (int j = 0; j < NS; ++j) {
+        double c[NLP];
 #pragma unroll
-        for (int j = NS - 1; j >= 1; --j) {
-            const double t = fma(s2, b1, __ldg(c + i * NS + j) - b2);
-            b2 = b1;
-            b1 = t;
-        }
-        g[i] = fma(s, b1, __ldg(c + i * NS) - b2);
+        for (int i = 0; i < NLP; i += 2) { const double2 t = ld2(m + j * NLP + i); c[i] = t.x; c[i + 1] = t.y; }
+        double v = c[NL - 1];
+#pragma unroll
+        for (int i = NL - 2; i >= 0; --i) v = fma(v, mu, c[i]);
+        col[j] = v;
     }
-    const double m2 = 2.0 * mu;
-    double b1 = 0.0, b2 = 0.0;
-#pragma unroll
-    for (int i = NL - 1; i >= 1; --i) {
-        const double t = fma(m2, b1, g[i] - b2);
-        b2 = b1;
-        b1 = t;
-    }
-    return fma(mu, b1, g[0] - b2);
+    return estrin<NS>(col, s);
 }
 
 // Closed-form cross terms of the top min(nq, 32) queue entries (one per lane), plus their
@@ -812,7 +821,7 @@ __device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmem &S, cons
             double l2k = lam * lam;
 #pragma unroll
             for (int i = 0; i < K; ++i) l2k *= lam * lam;
-            part = l2k * cheb2d<X::NL, X::NS>(xb + 6 + (lo ? 0 : X::NP), 2.0 * lam - 1.0, sv);
+            part = l2k * mono2d<X::NL, X::NLP, X::NS>(xb + 6 + (lo ? 0 : X::NP), 2.0 * lam - 1.0, sv);
             if (COUNT) ++c_poly;
         }
         const double I11 = sy == 0 ? (inside ? part : (below_all ? full : 0.0))

@@ -24,7 +24,7 @@ if os.environ.get("SIAC_LIB_VARIANT"):
     LIB_PATH = os.path.join(_HERE, f"libsiac_b200.{os.environ['SIAC_LIB_VARIANT']}.so")
 SOURCES = [os.path.join(_HERE, "csrc", f) for f in (
     "siac.cu", "siac_eval_k.cu", "siac_internal.h", "siac_device.cuh", "siac_tile.cuh", "siac_ws.cuh",
-    "siac_clipfast.cuh", "siac_jump.cuh", "siac_math.cpp", "siac_math.h", "siac_quadrature.h")]
+    "siac_clipfast.cuh", "siac_jump.cuh", "siac_math.cpp", "siac_math.h", "siac_quadrature.h", "siac_io.cu")]
 SOURCES.append(os.path.join(os.path.dirname(_HERE), "include", "siac.h"))
 
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
@@ -53,6 +53,8 @@ def build(force: bool = False, verbose: bool = False, extra_flags=(), out_path: 
     part_deps = {0: cs("siac_jump.cuh"), 1: [], 2: cs("siac_tile.cuh", "siac_clipfast.cuh"), 3: cs("siac_ws.cuh")}
     jobs = [(["g++", "-O2", "-std=c++17", "-fPIC", "-c", "-o", os.path.join(objdir, "siac_math.o")] + cs("siac_math.cpp"),
              os.path.join(objdir, "siac_math.o"), cs("siac_math.cpp", "siac_math.h"))]
+    jobs.append(([nvcc] + flags + ["-c", "-o", os.path.join(objdir, "siac_io.o")] + cs("siac_io.cu"),
+                 os.path.join(objdir, "siac_io.o"), cs("siac_io.cu", "siac_internal.h", "siac_math.h") + [SOURCES[-1]]))
     jobs.append(([nvcc] + flags + ["-c", "-o", os.path.join(objdir, "siac.o")] + cs("siac.cu"),
                  os.path.join(objdir, "siac.o"), cs("siac.cu", "siac_jump.cuh", "siac_math.h") + common))
     for k in (1, 2, 3, 4):
@@ -152,6 +154,14 @@ def lib():
         L.siac_last_error.argtypes = [vp]
         L.siac_version.restype = ctypes.c_char_p
         L.siac_version.argtypes = []
+        L.siac_projection_rule.restype = ctypes.c_int
+        L.siac_projection_rule.argtypes = [I32, D, D]
+        L.siac_map_points_async.restype = ctypes.c_int
+        L.siac_map_points_async.argtypes = [vp, vp, I64, vp, I32, vp, vp]
+        L.siac_project_async.restype = ctypes.c_int
+        L.siac_project_async.argtypes = [I32, I32, vp, I64, vp, vp]
+        L.siac_error_norms_async.restype = ctypes.c_int
+        L.siac_error_norms_async.argtypes = [vp, vp, vp, I64, vp, vp]
         _lib = L
     return _lib
 
@@ -159,7 +169,8 @@ def lib():
 EXPORTED = ["siac_create", "siac_eval", "siac_eval_async", "siac_set_counting", "siac_stats",
             "siac_set_schedule", "siac_set_timing", "siac_timing", "siac_probe_fp64",
             "siac_info", "siac_host_tables", "siac_debug_records",
-            "siac_destroy", "siac_last_error", "siac_version"]
+            "siac_destroy", "siac_last_error", "siac_version",
+            "siac_projection_rule", "siac_map_points_async", "siac_project_async", "siac_error_norms_async"]
 
 
 def _dp(a):
@@ -302,3 +313,40 @@ def probe_fp64(device: int = 0) -> float:
 
 def version() -> str:
     return lib().siac_version().decode()
+
+
+# ---------------------------------------------------------------- steps either side of the path
+# (SURVEY §8(f) NEXT-3): argument marshalling only; every step runs in csrc/siac_io.cu.
+
+def _ptr(t):
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _stream_ptr(stream):
+    return ctypes.c_void_p(0 if stream is None else stream.cuda_stream)
+
+
+def projection_rule(n_quad: int):
+    """(rs (n_quad^2, 2) unit-triangle nodes, w (n_quad^2,) reference-triangle weights)."""
+    rs = np.empty((n_quad * n_quad, 2))
+    w = np.empty(n_quad * n_quad)
+    _check(lib().siac_projection_rule(int(n_quad), _dp(rs), _dp(w)), None)
+    return rs, w
+
+
+def map_points_async(d_V, d_T, d_rs, d_out, stream=None) -> None:
+    """d_out[(t, q)] = v0 + r_q (v1 - v0) + s_q (v2 - v0); torch CUDA tensors (f64 / int32)."""
+    _check(lib().siac_map_points_async(_ptr(d_V), _ptr(d_T), int(d_T.shape[0]), _ptr(d_rs), int(d_rs.shape[0]),
+                                       _ptr(d_out), _stream_ptr(stream)), None)
+
+
+def project_async(k: int, n_quad: int, d_f, d_coeffs, stream=None) -> None:
+    """Orthonormal Dubiner modes (n_triangles, nb) of f sampled at the projection rule nodes."""
+    _check(lib().siac_project_async(int(k), int(n_quad), _ptr(d_f), int(d_coeffs.shape[0]), _ptr(d_coeffs),
+                                    _stream_ptr(stream)), None)
+
+
+def error_norms_async(d_u, d_ref, d_w, d_out, stream=None) -> None:
+    """d_out[0:3] = sqrt(sum w e^2), max |e|, sum w for e = u - ref (d_w may be None)."""
+    _check(lib().siac_error_norms_async(_ptr(d_u), _ptr(d_ref), None if d_w is None else _ptr(d_w),
+                                        int(d_u.shape[0]), _ptr(d_out), _stream_ptr(stream)), None)
