@@ -229,7 +229,7 @@ def run_siac(args):
     cands, pairs, pieces, subtris, corners, crosses, xsub, xpoly = allreduce_sum_int(
         [st["candidates"], st["pairs"], st["pieces"], st["subtris"], st["corner_terms"], st["cross_terms"],
          st["cross_subtris"], st["cross_polys"]])
-    jump = args.schedule in (0, 4, 5)
+    jump = args.schedule in (0, 4, 5, 6)
     if jump:
         # JUMP: its own algorithmic flops; general-path pairs (h < triangle size only) add
         # their clip-and-integrate sub-triangles at the direct method's rate
@@ -361,7 +361,7 @@ def run_siac(args):
                                             "direct SH + fan + quadrature (SURVEY §8(d))")},
                 "e2e": {"value": e2e_val, "unit": "points/s", "h2d_bytes_per_step": int(w.n_points * 16),
                         "d2h_bytes_per_step": int(w.n_points * 8)},
-                "schedule": ["default(jump-x)", "point", "tile", "ws", "jump", "jump-x"][args.schedule],
+                "schedule": ["default(jump-x)", "point", "tile", "ws", "jump", "jump-x", "elem"][args.schedule],
                 "gpu_launches": 2 * args.steps,
                 "gpu_launches_note": "per step and rank: k_point_keys + k_eval (ours) + CUB radix-sort kernels",
                 "clocks": clk}
@@ -393,7 +393,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--schedule", type=int, default=0,
                     help="0 = default (jump-x), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, "
-                         "4 = jump, 5 = jump with closed-form cross terms")
+                         "4 = jump, 5 = jump with closed-form cross terms, 6 = per-element (scatter)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-direct-count", dest="direct_count", action="store_false",
                     help="skip the (untimed) direct-decomposition count run")

@@ -137,13 +137,19 @@ siac_status siac_eval_async(siac_ctx *ctx, const double *d_points_xy, int64_t n_
  *                         clipped by the y knot line is the homothetic image of a fixed reference
  *                         corner clipped by a horizontal line, whose integral is a polynomial in
  *                         (homothety ratio, line height) on each of two height intervals, built
- *                         per triangle at create time (Chebyshev interpolation of exact samples). */
+ *                         per triangle at create time (Chebyshev interpolation of exact samples);
+ *   SIAC_SCHEDULE_ELEM    (6) the paper's per-element method (Alg. 3) on the JUMPX
+ *                         decomposition: one warp per triangle walks the point grid within its
+ *                         Eq. (3) bounds (L434-498), lane = candidate point, and scatter-adds each
+ *                         pair's contribution (atomics: the summation order, hence the last bits,
+ *                         varies between runs; every other schedule is bitwise deterministic). */
 #define SIAC_SCHEDULE_DEFAULT 0
 #define SIAC_SCHEDULE_POINT 1
 #define SIAC_SCHEDULE_TILE 2
 #define SIAC_SCHEDULE_WS 3
 #define SIAC_SCHEDULE_JUMP 4
 #define SIAC_SCHEDULE_JUMPX 5
+#define SIAC_SCHEDULE_ELEM 6
 siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule);
 
 /* Enable (1) / disable (0) geometry counting in later evaluations (adds atomics; off by default). */

@@ -45,6 +45,7 @@ struct siac_ctx {
     double *d_rec = nullptr;
     double *d_jrec = nullptr;    // schedule JUMP records (siac_jump.cuh)
     double *d_xrec = nullptr;    // closed-form cross-term polynomials (schedule JUMP-X)
+    int *d_pcell = nullptr;      // schedule ELEM: point CSR by row-major binning cell
     double4 *d_bbox = nullptr;
     int *d_cell_start = nullptr;
     double *d_kc = nullptr;
@@ -57,7 +58,7 @@ struct siac_ctx {
     int64_t cap_host = 0;
     double *d_hpts = nullptr, *d_hout = nullptr;
     // counters
-    int schedule = 0;            // 0 = default (= 5), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump, 5 = jump-x
+    int schedule = 0;            // 0 = default (= 5), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump, 5 = jump-x, 6 = per-element
     int *d_tile_counter = nullptr;
     int num_sms = 148;
     bool counting = false;
@@ -187,7 +188,8 @@ __device__ __forceinline__ double wrap_coord(double v, double lo, double L) {
 }
 
 __global__ void k_point_keys(const double *pts, int64_t np, double x0, double y0, double Lx, double Ly,
-                             int periodic, double cw, double chh, int ncx, int ncy, uint32_t *key, int *idx) {
+                             int periodic, double cw, double chh, int ncx, int ncy, uint32_t *key, int *idx,
+                             int rowmajor) {
     int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= np) return;
     double x = pts[2 * i], y = pts[2 * i + 1];
@@ -195,7 +197,7 @@ __global__ void k_point_keys(const double *pts, int64_t np, double x0, double y0
     if (periodic & 2) y = wrap_coord(y, y0, Ly);
     int cx = (int)fmin(fmax(floor((x - x0) / cw), 0.0), (double)(ncx - 1));
     int cy = (int)fmin(fmax(floor((y - y0) / chh), 0.0), (double)(ncy - 1));
-    key[i] = spread16((uint32_t)cx) | (spread16((uint32_t)cy) << 1);
+    key[i] = rowmajor ? (uint32_t)cy * (uint32_t)ncx + (uint32_t)cx : spread16((uint32_t)cx) | (spread16((uint32_t)cy) << 1);
     idx[i] = (int)i;
 }
 
@@ -230,19 +232,35 @@ void eval_device(siac_ctx *c, const double *d_pts, int64_t np, double *d_out, cu
     need(np <= (int64_t)0x7fffffff, "n_points must be < 2^31");
     ensure_scratch(c, np);
     const double Lx = c->dom[2] - c->dom[0], Ly = c->dom[3] - c->dom[1];
+    const bool elem = c->schedule == 6;          // per-element: points in row-major cell order
     k_point_keys<<<nblk(np, 256), 256, 0, st>>>(d_pts, np, c->dom[0], c->dom[1], Lx, Ly, c->periodic, c->cw,
-                                                c->chh, c->ncx, c->ncy, c->d_keys[0], c->d_idx[0]);
+                                                c->chh, c->ncx, c->ncy, c->d_keys[0], c->d_idx[0], elem ? 1 : 0);
     CK(cudaGetLastError());
     cub::DoubleBuffer<uint32_t> kb(c->d_keys[0], c->d_keys[1]);
     cub::DoubleBuffer<int> vb(c->d_idx[0], c->d_idx[1]);
     int end_bit = 1;
     while ((1ull << end_bit) <= (unsigned long long)std::max(c->ncx, c->ncy) && end_bit < 16) ++end_bit;
-    CK(cub::DeviceRadixSort::SortPairs(c->d_cub, c->cub_bytes, kb, vb, (int)np, 0, 2 * end_bit, st));
+    int key_bits = 2 * end_bit;
+    if (elem) {
+        key_bits = 1;
+        while ((1ull << key_bits) < (unsigned long long)c->ncx * c->ncy && key_bits < 32) ++key_bits;
+    }
+    CK(cub::DeviceRadixSort::SortPairs(c->d_cub, c->cub_bytes, kb, vb, (int)np, 0, key_bits, st));
     EvalArgs a;
     a.pts = d_pts; a.perm = vb.Current(); a.np = np; a.out = d_out;
     a.rec = c->d_rec; a.jrec = c->d_jrec; a.xrec = c->d_xrec; a.bbox = c->d_bbox; a.cell_start = c->d_cell_start;
     a.kc = c->d_kc;
     a.xpoly = (c->schedule == 0 || c->schedule == 5) ? 1 : 0;
+    a.nt = c->nt;
+    a.pcell_start = nullptr;
+    if (elem) {
+        const int64_t ncell = (int64_t)c->ncx * c->ncy;
+        if (!c->d_pcell) CK(cudaMalloc(&c->d_pcell, sizeof(int) * (ncell + 1)));
+        k_cell_start<<<nblk(ncell + 1, 256), 256, 0, st>>>(kb.Current(), np, ncell, c->d_pcell);
+        CK(cudaGetLastError());
+        CK(cudaMemsetAsync(d_out, 0, sizeof(double) * np, st));    // the pairs scatter-add
+        a.pcell_start = c->d_pcell;
+    }
     a.x0 = c->dom[0]; a.y0 = c->dom[1]; a.Lx = Lx; a.Ly = Ly;
     a.h = c->h; a.inv_h = c->inv_h; a.hw = 0.5 * (3 * c->k + 1) * c->h;
     a.cw = c->cw; a.chh = c->chh; a.ex = c->ex; a.ey = c->ey;
@@ -269,7 +287,10 @@ void eval_device(siac_ctx *c, const double *d_pts, int64_t np, double *d_out, cu
         {siac_launch_eval_k4_p0, siac_launch_eval_k4_p1, siac_launch_eval_k4_p2, siac_launch_eval_k4_p3}};
     if (c->k < 1 || c->k > 4) throw Fail{SIAC_EINTERNAL, "bad k"};
     const int part = (c->schedule == 0 || c->schedule >= 4) ? 0 : c->schedule;
-    const cudaError_t e = table[c->k - 1][part](a, c->counting, c->d_tile_counter, c->num_sms, st);
+    static const siac_launch_fn elem_table[4] = {siac_launch_elem_k1, siac_launch_elem_k2, siac_launch_elem_k3,
+                                                 siac_launch_elem_k4};
+    const cudaError_t e = elem ? elem_table[c->k - 1](a, c->counting, c->d_tile_counter, c->num_sms, st)
+                               : table[c->k - 1][part](a, c->counting, c->d_tile_counter, c->num_sms, st);
     CK(e);
     CK(cudaGetLastError());
     if (ev_stop) CK(cudaEventRecord(ev_stop, st));
@@ -295,7 +316,7 @@ void free_ctx(siac_ctx *c) {
     if (!c) return;
     cudaSetDevice(c->device);
     for (auto &e : c->ev) { cudaEventDestroy(e.first); cudaEventDestroy(e.second); }
-    void *ptrs[] = {c->d_rec, c->d_jrec, c->d_xrec, c->d_bbox, c->d_cell_start, c->d_kc, c->d_keys[0], c->d_keys[1],
+    void *ptrs[] = {c->d_rec, c->d_jrec, c->d_xrec, c->d_pcell, c->d_bbox, c->d_cell_start, c->d_kc, c->d_keys[0], c->d_keys[1],
                     c->d_idx[0], c->d_idx[1], c->d_cub, c->d_hpts, c->d_hout, c->d_cnt, c->d_tile_counter};
     for (void *p : ptrs)
         if (p) cudaFree(p);
@@ -560,7 +581,7 @@ siac_status siac_stats(siac_ctx *ctx, siac_counters *out) {
 
 siac_status siac_set_schedule(siac_ctx *ctx, int32_t schedule) {
     if (!ctx) { g_err = "NULL context"; return SIAC_EINVAL; }
-    if (schedule < 0 || schedule > 5) { ctx->err = "unknown schedule"; return SIAC_EINVAL; }
+    if (schedule < 0 || schedule > 6) { ctx->err = "unknown schedule"; return SIAC_EINVAL; }
     ctx->schedule = schedule;
     return SIAC_OK;
 }

@@ -223,4 +223,20 @@ cudaError_t SIAC_CAT(siac_prep_cross_k, SIAC_K)(const double *jrec, int64_t nt, 
     return cudaGetLastError();
 }
 int SIAC_CAT(siac_xrec_doubles_k, SIAC_K)() { return siacjump::XRec<SIAC_K>::RS; }
+cudaError_t SIAC_CAT(siac_launch_elem_k, SIAC_K)(const EvalArgs &a, bool count, int *, int, cudaStream_t st) {
+    if (a.nt == 0) return cudaSuccess;
+    siacjump::JumpArgs j;
+    j.pts = a.pts; j.perm = a.perm; j.np = a.np; j.out = a.out; j.rec = a.rec; j.jrec = a.jrec; j.xrec = a.xrec;
+    j.pcell_start = a.pcell_start; j.bbox = a.bbox; j.cell_start = a.cell_start; j.kc = a.kc;
+    j.x0 = a.x0; j.y0 = a.y0; j.Lx = a.Lx; j.Ly = a.Ly; j.inv_h = a.inv_h; j.hw = a.hw; j.cw = a.cw; j.chh = a.chh;
+    j.ex = a.ex; j.ey = a.ey; j.ncx = a.ncx; j.ncy = a.ncy; j.periodic = a.periodic; j.cnt = a.cnt;
+    const unsigned grid = (unsigned)((a.nt + siacjump::WARPS - 1) / siacjump::WARPS);
+    const bool gen = std::max(a.ex, a.ey) > a.h * (1.0 + 1e-9);
+    constexpr int K = SIAC_K;
+    if (count) { if (gen) siacjump::k_eval_elem<K, true, true><<<grid, siacjump::WARPS * 32, 0, st>>>(j, a.nt);
+                 else siacjump::k_eval_elem<K, true, false><<<grid, siacjump::WARPS * 32, 0, st>>>(j, a.nt); }
+    else { if (gen) siacjump::k_eval_elem<K, false, true><<<grid, siacjump::WARPS * 32, 0, st>>>(j, a.nt);
+           else siacjump::k_eval_elem<K, false, false><<<grid, siacjump::WARPS * 32, 0, st>>>(j, a.nt); }
+    return cudaGetLastError();
+}
 #endif

@@ -24,6 +24,8 @@ struct EvalArgs {            // arguments of every evaluation schedule
     double cw, chh, ex, ey;
     int ncx, ncy, periodic;
     int xpoly;                // jump schedule: 1 = closed-form cross terms, 0 = clipped + quadrature
+    const int *pcell_start;   // schedule ELEM: point CSR by row-major binning cell
+    int64_t nt;               // number of triangles
     unsigned long long *cnt;  // [candidates, pairs, pieces, subtris, corner, cross, cross_subtris, cross_polys]
 };
 
@@ -35,6 +37,7 @@ struct EvalArgs {            // arguments of every evaluation schedule
     SIAC_DECL_KP(k, 0) SIAC_DECL_KP(k, 1) SIAC_DECL_KP(k, 2) SIAC_DECL_KP(k, 3)                 \
     cudaError_t siac_prep_jump_k##k(const double *rec, int64_t nt, double h, double *jrec);        \
     cudaError_t siac_prep_cross_k##k(const double *jrec, int64_t nt, double *xrec);                \
+    cudaError_t siac_launch_elem_k##k(const EvalArgs &a, bool count, int *, int, cudaStream_t st); \
     int siac_xrec_doubles_k##k();
 SIAC_DECL_K(1)
 SIAC_DECL_K(2)

@@ -388,6 +388,7 @@ struct JumpArgs {
     const double *rec;        // Rec<K> (general fallback)
     const double *jrec;       // JRec<K>
     const double *xrec;       // XRec<K> (closed-form cross terms)
+    const int *pcell_start;   // schedule ELEM: CSR of the points sorted by row-major binning cell
     const double4 *bbox;
     const int *cell_start;
     const double *kc;
@@ -762,6 +763,51 @@ __device__ __forceinline__ double mono2d(const double *m, double mu, double s) {
     return estrin<NS>(col, s);
 }
 
+// I11 / (sgn alpha_x sgn alpha_y): \int_{x corner ∩ y corner} (z1 - X)^K (z2 - Y)^K u for the x
+// corner of side sx with homothety ratio lam, the y knot Y (zeta frame) and the y corner on side
+// sy; xb = the triangle's XRec block of side sx.  poly: evaluated by an interval polynomial.
+template <int K>
+__device__ __forceinline__ double cross_I11(const double *jr, const double *xb, double lam, double Y, int sx, int sy,
+                                            bool &poly) {
+    using J = JRec<K>;
+    using X = XRec<K>;
+    const double Ay = __ldg(jr + J::OFF_GEO + (sx == 0 ? 5 : 1));
+    const double2 v01 = ld2(xb), v2i = ld2(xb + 2), i1 = ld2(xb + 4);
+    const double Yp = fma(Y - Ay, 1.0 / lam, Ay);     // the y knot in the reference corner's frame
+    const bool above_all = Yp >= v2i.x;                // the line is above the corner
+    const bool below_all = Yp <= v01.x;                // ... below it
+    // the full-corner integral of (z1 - X)^K (z2 - Y)^K u: corner polynomials with the
+    // coefficients of (zeta2 - Y)^K in powers of zeta2
+    const bool need_full = sy == 0 ? below_all : !below_all;
+    double full = 0.0;
+    if (need_full) {
+        double cy[K + 1];
+        double pw = 1.0;
+#pragma unroll
+        for (int b = K; b >= 0; --b) {      // C(K, b) (-Y)^{K-b}
+            double bin = 1.0;
+#pragma unroll
+            for (int r = 0; r < K - b; ++r) bin = bin * (double)(K - r) / (double)(r + 1);
+            cy[b] = bin * pw;
+            pw *= -Y;
+        }
+        full = corner_eval<K>(jr + J::OFF_G + sx * J::NGP, cy, lam);
+    }
+    double part = 0.0;                                 // lambda^{2K+2} F_above(lambda, Y')
+    const bool inside = !above_all && !below_all;
+    if (inside) {
+        const bool lo = Yp < v01.y;
+        const double va = lo ? v01.x : v01.y, iw = lo ? v2i.y : i1.x;
+        const double sv = fma(2.0 * (Yp - va), iw, -1.0);
+        double l2k = lam * lam;
+#pragma unroll
+        for (int i = 0; i < K; ++i) l2k *= lam * lam;
+        part = l2k * mono2d<X::NL, X::NLP, X::NS>(xb + 6 + (lo ? 0 : X::NP), 2.0 * lam - 1.0, sv);
+    }
+    poly = inside;
+    return sy == 0 ? (inside ? part : (below_all ? full : 0.0)) : (inside ? full - part : (above_all ? full : 0.0));
+}
+
 // Closed-form cross terms of the top min(nq, 32) queue entries (one per lane), plus their
 // deferred y-corner terms, added to the owners' accumulators.
 template <int K, bool COUNT>
@@ -786,46 +832,12 @@ __device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmem &S, cons
         double pc[K + 1];
         base_taylor<K>(kcp, rowx, S.qE[e], pc);
         const double ycorner = ay * corner_eval<K>(jr + J::OFF_G + (2 + sy) * J::NGP, pc, S.qL[e]);
-        // the x corner's homothety ratio and the y knot in the reference corner's frame
+        // the x corner's homothety ratio
         const double2 lh = ld2(jr + J::OFF_AX), iv = ld2(jr + J::OFF_AX + 4);
         const double lam = sx == 0 ? (lh.y - Xk) * iv.y : (Xk - lh.x) * iv.x;
-        const double Ay = __ldg(jr + J::OFF_GEO + (sx == 0 ? 5 : 1));
-        const double *xb = a.xrec + (int64_t)X::RS * tri + sx * X::XB;
-        const double2 v01 = ld2(xb), v2i = ld2(xb + 2), i1 = ld2(xb + 4);
-        const double Yp = fma(Y - Ay, 1.0 / lam, Ay);
-        const bool above_all = Yp >= v2i.x;      // the line is above the corner
-        const bool below_all = Yp <= v01.x;      // ... below it
-        // the full-corner integral of (z1 - X)^K (z2 - Y)^K u: corner polynomials with the
-        // coefficients of (zeta2 - Y)^K in powers of zeta2
-        const bool need_full = sy == 0 ? below_all : !below_all;
-        double full = 0.0;
-        if (need_full) {
-            double cy[K + 1];
-            double pw = 1.0;
-#pragma unroll
-            for (int b = K; b >= 0; --b) {      // C(K, b) (-Y)^{K-b}
-                double bin = 1.0;
-#pragma unroll
-                for (int r = 0; r < K - b; ++r) bin = bin * (double)(K - r) / (double)(r + 1);
-                cy[b] = bin * pw;
-                pw *= -Y;
-            }
-            full = corner_eval<K>(jr + J::OFF_G + sx * J::NGP, cy, lam);
-        }
-        double part = 0.0;               // lambda^{2K+2} F_above(lambda, Y')
-        const bool inside = !above_all && !below_all;
-        if (inside) {
-            const bool lo = Yp < v01.y;
-            const double va = lo ? v01.x : v01.y, iw = lo ? v2i.y : i1.x;
-            const double sv = fma(2.0 * (Yp - va), iw, -1.0);
-            double l2k = lam * lam;
-#pragma unroll
-            for (int i = 0; i < K; ++i) l2k *= lam * lam;
-            part = l2k * mono2d<X::NL, X::NLP, X::NS>(xb + 6 + (lo ? 0 : X::NP), 2.0 * lam - 1.0, sv);
-            if (COUNT) ++c_poly;
-        }
-        const double I11 = sy == 0 ? (inside ? part : (below_all ? full : 0.0))
-                                   : (inside ? full - part : (above_all ? full : 0.0));
+        bool poly = false;
+        const double I11 = cross_I11<K>(jr, a.xrec + (int64_t)X::RS * tri + sx * X::XB, lam, Y, sx, sy, poly);
+        if (COUNT && poly) ++c_poly;
         val = fma(ax * ay, I11, ycorner);
     }
     nq -= take;
@@ -1084,6 +1096,125 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
             if (i == 2 || i == 3 || i == 4 || i == 7) {
                 for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(0xffffffffu, x, o);
             }
+            if (lane == 0 && x) atomicAdd(a.cnt + i, x);
+        }
+    }
+}
+
+
+// ------------------------------------------------------------------ per-element schedule (ELEM)
+// The paper's per-element method (Alg. 3; search bounds Eq. (3))
+// on the same exact decomposition: one warp per triangle (cell order), its stencil-expanded
+// bounding box walked over the point grid (row runs of the row-major point CSR, periodic images
+// unwrapped), 32 candidate points per step (lane = point), the whole pair contribution --
+// moments, both corner terms, the closed-form cross term -- evaluated from the one triangle's
+// record (broadcast loads), and scattered to the point with one atomic add per pair (the
+// paper's per-patch partial solutions + reduction, L636-652, become atomics; the summation
+// order, hence the last bits, is not fixed).
+template <int K, bool COUNT, bool GEN>
+__global__ void __launch_bounds__(WARPS * 32) k_eval_elem(JumpArgs a, int64_t nt) {
+    using J = JRec<K>;
+    using X = XRec<K>;
+    constexpr int NC = 3 * K + 1;
+    __shared__ double kcp[(NC + 2) * (K + 1)];
+    __shared__ double alpha[NC + 1];
+    for (int i = threadIdx.x; i < (NC + 2) * (K + 1); i += blockDim.x) {
+        const int row = i / (K + 1);
+        kcp[i] = (row == 0 || row == NC + 1) ? 0.0 : a.kc[i - (K + 1)];
+    }
+    __syncthreads();
+    for (int m = threadIdx.x; m <= NC; m += blockDim.x) alpha[m] = kcp[(m + 1) * (K + 1) + K] - kcp[m * (K + 1) + K];
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int64_t t = (int64_t)blockIdx.x * WARPS + (threadIdx.x >> 5);
+    if (t >= nt) return;                           // warp-uniform
+    const double *jr = a.jrec + (int64_t)J::RS * t;
+    const double4 tb = a.bbox[t];
+    // Eq. (3) per-element bounds: floor((min - w/2)/c_e) .. floor((max + w/2)/c_e)
+    int C0 = (int)floor((tb.x - a.hw - a.x0) / a.cw), C1 = (int)floor((tb.z + a.hw - a.x0) / a.cw);
+    int R0 = (int)floor((tb.y - a.hw - a.y0) / a.chh), R1 = (int)floor((tb.w + a.hw - a.y0) / a.chh);
+    if (!(a.periodic & 2)) { R0 = max(R0, 0); R1 = min(R1, a.ncy - 1); }
+    if (!(a.periodic & 1)) { C0 = max(C0, 0); C1 = min(C1, a.ncx - 1); }
+    const double2 cen = ld2(jr);
+    constexpr double MT0 = 0.5 * (3 * K + 1);
+    unsigned long long c_cand = 0, c_pairs = 0, c_pieces = 0, c_sub = 0, c_corner = 0, c_cross = 0, c_poly = 0;
+    for (int R = R0; R <= R1; ++R) {
+        int r = R, qy = 0;
+        if (a.periodic & 2) { r = ((R % a.ncy) + a.ncy) % a.ncy; qy = (R - r) / a.ncy; }
+        const double rsy = -qy * a.Ly;          // triangle image relative to the wrapped points
+        int C = C0;
+        while (C <= C1) {
+            int c = C, qx = 0;
+            if (a.periodic & 1) { c = ((C % a.ncx) + a.ncx) % a.ncx; qx = (C - c) / a.ncx; }
+            const int cend = (a.periodic & 1) ? min(C1, (qx + 1) * a.ncx - 1) : C1;
+            const double rsx = -qx * a.Lx;
+            const int p_beg = __ldg(a.pcell_start + r * a.ncx + c);
+            const int p_end = __ldg(a.pcell_start + r * a.ncx + c + (cend - C) + 1);
+            C = cend + 1;
+            const double bx0 = tb.x + rsx, bx1 = tb.z + rsx, by0 = tb.y + rsy, by1 = tb.w + rsy;
+            for (int p0 = p_beg; p0 < p_end; p0 += 32) {
+                const int sp = p0 + lane;
+                const bool valid = sp < p_end;
+                int orig = 0;
+                double x1 = 0.0, x2 = 0.0;
+                if (valid) {
+                    orig = a.perm[sp];
+                    x1 = a.pts[2 * (int64_t)orig];
+                    x2 = a.pts[2 * (int64_t)orig + 1];
+                    if (a.periodic & 1) { x1 = x1 - a.Lx * floor((x1 - a.x0) / a.Lx); if (x1 >= a.x0 + a.Lx) x1 -= a.Lx; if (x1 < a.x0) x1 = a.x0; }
+                    if (a.periodic & 2) { x2 = x2 - a.Ly * floor((x2 - a.y0) / a.Ly); if (x2 >= a.y0 + a.Ly) x2 -= a.Ly; if (x2 < a.y0) x2 = a.y0; }
+                }
+                const bool hit = valid && (bx0 < x1 + a.hw && bx1 > x1 - a.hw && by0 < x2 + a.hw && by1 > x2 - a.hw);
+                if (COUNT) { c_cand += valid; c_pairs += hit; }
+                if (!__any_sync(0xffffffffu, hit)) continue;
+                const double dx = fma((cen.x + rsx) - x1, a.inv_h, MT0);
+                const double dy = fma((cen.y + rsy) - x2, a.inv_h, MT0);
+                const Cut cx = axis_cut<K, GEN>(jr + J::OFF_AX, dx);
+                const Cut cy = axis_cut<K, GEN>(jr + J::OFF_AX + 6, dy);
+                double v = 0.0;
+                if (GEN && (cx.multi || cy.multi)) {
+                    if (hit) {
+                        const GenOut go = general_pair<K, COUNT>(a.rec, kcp, (int)t, rsx, rsy, x1, x2, a.inv_h);
+                        v = go.v;
+                        if (COUNT) { c_pieces += go.pieces; c_sub += go.subtris; }
+                    }
+                } else {
+                    double p[K + 1], q[K + 1];
+                    base_taylor<K>(kcp, cx.row, cx.e, p);
+                    base_taylor<K>(kcp, cy.row, cy.e, q);
+                    double ve = 0.0, vo = 0.0;
+#pragma unroll
+                    for (int aa = K; aa >= 0; --aa) {
+                        double sacc = 0.0;
+#pragma unroll
+                        for (int bb = K; bb >= 0; --bb) sacc = fma(q[bb], __ldg(jr + J::OFF_MU + aa * (K + 1) + bb), sacc);
+                        if (aa & 1) vo = fma(p[aa], sacc, vo);
+                        else ve = fma(p[aa], sacc, ve);
+                    }
+                    v = ve + vo;
+                    const double ax = cx.cut ? (cx.side == 0 ? alpha[cx.m] : -alpha[cx.m]) : 0.0;
+                    const double ay = cy.cut ? (cy.side == 0 ? alpha[cy.m] : -alpha[cy.m]) : 0.0;
+                    if (cx.cut) v = fma(ax, corner_eval<K>(jr + J::OFF_G + cx.side * J::NGP, q, cx.lam), v);
+                    if (cy.cut) v = fma(ay, corner_eval<K>(jr + J::OFF_G + (2 + cy.side) * J::NGP, p, cy.lam), v);
+                    if (cx.cut && cy.cut) {
+                        bool poly = false;
+                        const double I11 = cross_I11<K>(jr, a.xrec + (int64_t)X::RS * t + cx.side * X::XB, cx.lam, cy.X,
+                                                        cx.side, cy.side, poly);
+                        v = fma(ax * ay, I11, v);
+                        if (COUNT && hit) { ++c_cross; c_poly += poly; }
+                    }
+                    if (COUNT && hit) c_corner += (int)cx.cut + (int)cy.cut;
+                }
+                if (hit) atomicAdd(a.out + orig, v);
+            }
+        }
+    }
+    if (COUNT) {
+        unsigned long long vv[8] = {c_cand, c_pairs, c_pieces, c_sub, c_corner, c_cross, 0ull, c_poly};
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            unsigned long long x = vv[i];
+            for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(0xffffffffu, x, o);
             if (lane == 0 && x) atomicAdd(a.cnt + i, x);
         }
     }

@@ -247,7 +247,7 @@ class Context:
 
     def set_schedule(self, schedule: int) -> None:
         """0 = default (fastest = 5), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump,
-        5 = jump with closed-form cross terms."""
+        5 = jump with closed-form cross terms, 6 = per-element (the paper's Alg. 3 mapping, scatter-add)."""
         _check(lib().siac_set_schedule(self._ptr, int(schedule)), self._ptr)
 
     def set_timing(self, on: bool = True) -> None:

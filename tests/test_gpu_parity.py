@@ -80,7 +80,7 @@ def test_cfg2_every_point(siac_mod, oracle_mod, field):
 
 
 @pytest.mark.parametrize("c", [1, 2])
-@pytest.mark.parametrize("schedule", [1, 2, 3, 4, 5])
+@pytest.mark.parametrize("schedule", [1, 2, 3, 4, 5, 6])
 def test_every_schedule_matches_oracle(siac_mod, oracle_mod, c, schedule):
     """Every schedule (point, tile, warp-specialized, jump) computes the same values."""
     w = cfg(c, "random")
@@ -89,7 +89,7 @@ def test_every_schedule_matches_oracle(siac_mod, oracle_mod, c, schedule):
 
 
 @pytest.mark.parametrize("k", [1, 2, 3, 4])
-@pytest.mark.parametrize("schedule", [2, 4, 5])
+@pytest.mark.parametrize("schedule", [2, 4, 5, 6])
 def test_every_k_delaunay_random_field(siac_mod, oracle_mod, k, schedule):
     """Every degree on an unstructured periodic mesh, random modes, h = max edge: the jump
     schedule's corner polynomials and cross terms at every k against the oracle."""
@@ -104,7 +104,7 @@ def test_every_k_delaunay_random_field(siac_mod, oracle_mod, k, schedule):
     assert_parity(g, oracle_mod.oracle_eval(V, T, C, k, h, P))
 
 
-@pytest.mark.parametrize("sch", [4, 5])
+@pytest.mark.parametrize("sch", [4, 5, 6])
 @pytest.mark.parametrize("c,m", [(3, 400), (4, 150)])
 def test_jump_and_tile_agree_large(siac_mod, oracle_mod, c, m, sch):
     """cfg 3 (graded) and cfg 4 (k = 4): the jump schedules against the oracle on a sample and
@@ -172,7 +172,7 @@ def test_counters_agree_between_schedules(siac_mod):
     ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
     ctx.set_counting(True)
     got = []
-    for sch in (2, 1, 3, 4, 5):
+    for sch in (2, 1, 3, 4, 5, 6):
         ctx.set_schedule(sch)
         ctx.eval(w.points)
         got.append(ctx.stats())
@@ -195,6 +195,10 @@ def test_counters_agree_between_schedules(siac_mod):
     assert (x["pairs"], x["corner_terms"], x["cross_terms"]) == (j["pairs"], j["corner_terms"], j["cross_terms"])
     assert x["pieces"] == 0 and x["subtris"] == 0 and x["cross_subtris"] == 0
     assert 0 < x["cross_polys"] <= x["cross_terms"]
+    e = got[5]      # per-element: the same pairs found from the other side (Eq. (3) element bounds)
+    assert (e["pairs"], e["corner_terms"], e["cross_terms"], e["cross_polys"]) == \
+        (x["pairs"], x["corner_terms"], x["cross_terms"], x["cross_polys"])
+    assert e["candidates"] >= e["pairs"]
 
 
 # ------------------------------------------------------------------ edge cases
