@@ -133,7 +133,8 @@ cudaError_t launch_part(const EvalArgs &a, bool count, int *, int, cudaStream_t 
     j.ncx = a.ncx; j.ncy = a.ncy; j.periodic = a.periodic; j.cnt = a.cnt;
     const int64_t ntiles = (a.np + 31) / 32;
     const unsigned grid = (unsigned)((ntiles + siacjump::WARPS - 1) / siacjump::WARPS);
-    const size_t smem = (sizeof(siacjump::WarpSmem) + sizeof(siacjump::WarpStage<K>)) * siacjump::WARPS;
+    const size_t smem = ((a.xpoly ? sizeof(siacjump::WarpSmemX) : sizeof(siacjump::WarpSmem)) +
+                         sizeof(siacjump::WarpStage<K>)) * siacjump::WARPS;
     // GEN: some triangle is wider than h (in x or y), so a pair may see two knots on an axis
     const bool gen = std::max(a.ex, a.ey) > a.h * (1.0 + 1e-9);
 #define SIAC_LAUNCH_JUMP(C, G, XP)                                                                             \

@@ -350,20 +350,23 @@ constexpr int WARPS = SIAC_JUMP_WARPS;
 constexpr int QCAP = 64;      // cross-term queue: < 32 left over + 32 new
 constexpr int SCAP = 96;      // staged cross sub-triangles: < 32 left over + <= 64 new
 
-struct WarpSmem {
+template <int SC> struct WarpSmemT {
     // cross-term queue (one entry per lane with a knot on both axes)
     int qtri[QCAP];
     int qinfo[QCAP];          // lane | sx << 5 | sy << 6 | mx << 7 | my << 12 | row_x << 17
     double qX[QCAP], qY[QCAP];
     double qE[QCAP], qL[QCAP]; // deferred y-corner term: base-x offset e_x, y homothety ratio
     // staged cross sub-triangles (compacted; integrated 32 at a time)
-    double s0x[SCAP], s0y[SCAP], s1x[SCAP], s1y[SCAP], s2x[SCAP], s2y[SCAP];
-    double sX[SCAP], sY[SCAP];
-    int stri[SCAP], sinfo[SCAP];
+    double s0x[SC], s0y[SC], s1x[SC], s1y[SC], s2x[SC], s2y[SC];
+    double sX[SC], sY[SC];
+    int stri[SC], sinfo[SC];
     double acc[32];
     double4 cbox[32];
     int klist[32];            // kept candidates of the current chunk (box meets the tile's stencils)
 };
+using WarpSmem = WarpSmemT<SCAP>;     // schedule JUMP: staged cross sub-triangles
+using WarpSmemX = WarpSmemT<2>;       // schedule JUMPX: no sub-triangles (smaller)
+template <bool XP> using WarpSmemFor = typename std::conditional<XP, WarpSmemX, WarpSmem>::type;
 
 #ifndef SIAC_JUMP_STAGES
 #define SIAC_JUMP_STAGES 2        // records in flight per warp (TMA ring)
@@ -616,7 +619,8 @@ __device__ __forceinline__ int warp_excl_scan(int v, int lane, int &total) {
 }
 
 // Sum v over lanes with equal key (keys >= 32 ignored), in lane order, into S.acc[key].
-__device__ __forceinline__ void seg_add(WarpSmem &S, int key, double v, int lane) {
+template <class SM_>
+__device__ __forceinline__ void seg_add(SM_ &S, int key, double v, int lane) {
     const unsigned grp = __match_any_sync(0xffffffffu, key);
     const int leader = __ffs(grp) - 1;
     double sum = (lane == leader) ? v : 0.0;
@@ -811,7 +815,7 @@ __device__ __forceinline__ double cross_I11(const double *jr, const double *xb, 
 // Closed-form cross terms of the top min(nq, 32) queue entries (one per lane), plus their
 // deferred y-corner terms, added to the owners' accumulators.
 template <int K, bool COUNT>
-__device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmem &S, const double *kcp, const double *alpha,
+__device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, const double *kcp, const double *alpha,
                                             int &nq, int lane, unsigned long long &c_poly) {
     using J = JRec<K>;
     using X = XRec<K>;
@@ -845,14 +849,18 @@ __device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmem &S, cons
     seg_add(S, key, val, lane);
 }
 
+#ifndef SIAC_JUMPX_MINB
+#define SIAC_JUMPX_MINB SIAC_JUMP_MINB
+#endif
 template <int K, bool COUNT, bool GEN, bool XP>
-__global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpArgs a) {
+__global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_MINB) k_eval_jump(JumpArgs a) {
     using J = JRec<K>;
     constexpr int NC = 3 * K + 1;
     __shared__ double kcp[(NC + 2) * (K + 1)];
     __shared__ double alpha[NC + 1];
     extern __shared__ __align__(16) unsigned char jump_dsm[];
-    WarpSmem *wsm = reinterpret_cast<WarpSmem *>(jump_dsm);
+    using WS = WarpSmemFor<XP>;
+    WS *wsm = reinterpret_cast<WS *>(jump_dsm);
     for (int i = threadIdx.x; i < (NC + 2) * (K + 1); i += blockDim.x) {
         const int row = i / (K + 1);
         kcp[i] = (row == 0 || row == NC + 1) ? 0.0 : a.kc[i - (K + 1)];
@@ -863,7 +871,7 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
 
     const int lane = threadIdx.x & 31;
     const int wid = threadIdx.x >> 5;
-    WarpSmem &S = wsm[wid];
+    WS &S = wsm[wid];
     WarpStage<K> &T = reinterpret_cast<WarpStage<K> *>(wsm + WARPS)[wid];
     const int64_t p0 = ((int64_t)blockIdx.x * WARPS + wid) * 32;
     if (p0 >= a.np) return;                       // warp-uniform
@@ -1054,7 +1062,7 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
             if (COUNT) c_cross += __popc(cm) * (lane == 0);
             __syncwarp();
             if (nq >= 32) {
-                if (XP) {
+                if constexpr (XP) {
                     cross_stage<K, COUNT>(a, S, kcp, alpha, nq, lane, c_xpoly);
                 } else {
                     clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
@@ -1063,12 +1071,12 @@ __global__ void __launch_bounds__(WARPS * 32, SIAC_JUMP_MINB) k_eval_jump(JumpAr
             }
         }
     });
-    if (XP) {
+    if constexpr (XP) {
         while (nq > 0) cross_stage<K, COUNT>(a, S, kcp, alpha, nq, lane, c_xpoly);
     } else {
         while (nq > 0) clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
+        while (ns > 0) integrate_stage<K>(a, S, alpha, ns, lane);
     }
-    while (ns > 0) integrate_stage<K>(a, S, alpha, ns, lane);
     __syncwarp();
     // second pass, only for tiles that met pairs with several knots on an axis (h smaller than
     // the triangles): those pairs take the clip-and-integrate path, out of the hot loop
