@@ -208,7 +208,8 @@ def run_siac(args):
     k = w.k
     if world > 1:
         from paper_conf_sc_0007k13_b200 import dist as sdist
-        part = sdist.partition(w.points, world)
+        wts = sdist.work_estimate(w.V, w.T, w.points, 0.5 * (3 * k + 1) * w.h)
+        part = sdist.partition(w.points, world, weights=wts)
         sub = sdist.local_problem(w.V, w.T, w.C, w.points, w.k, w.h, part, rank)
         V, T, C, P_local = sub["V"], sub["T"], sub["C"], sub["points"]
     else:

@@ -116,3 +116,32 @@ def test_gloo_dist_eval_matches_single_process(world, tmp_path, oracle_mod):
     w = inputs.make_config(1, field_kind="random")
     ref = oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, w.points)
     assert np.abs(got - ref).max() <= 1e-13 * np.abs(ref).max()
+
+
+def test_work_estimate_tracks_pair_counts_and_balances_graded_mesh():
+    """The per-point work proxy follows the exact number of (point, triangle image) box pairs
+    on the graded mesh (cfg 3), and partitioning by it balances the ranks' pairs where an
+    equal-count partition does not."""
+    w = inputs.make_config(3)
+    hw = 0.5 * (3 * w.k + 1) * w.h
+    est = sdist.work_estimate(w.V, w.T, w.points, hw)
+    rng = np.random.default_rng(5)
+    idx = rng.choice(w.n_points, 300, replace=False)
+    tx, ty = w.V[w.T][:, :, 0], w.V[w.T][:, :, 1]
+    exact = np.zeros(len(idx))
+    for n, i in enumerate(idx):
+        x = w.points[i]
+        for a in (-1, 0, 1):
+            for b in (-1, 0, 1):
+                exact[n] += np.count_nonzero((tx.min(1) + a < x[0] + hw) & (tx.max(1) + a > x[0] - hw) &
+                                             (ty.min(1) + b < x[1] + hw) & (ty.max(1) + b > x[1] - hw))
+    assert exact.max() > 3 * exact.min()                       # the mesh is graded
+    ratio = est[idx] / exact
+    assert np.std(ratio) / np.mean(ratio) < 0.1                # proportional to the pair count
+    world = 8          # (8 ranks: an equal-count cut is 2x out of balance on this mesh)
+    spread = {}
+    for name, wts in (("count", None), ("work", est)):
+        part = sdist.partition(w.points, world, weights=wts)
+        tot = [est[part["order"][part["bounds"][r]:part["bounds"][r + 1]]].sum() for r in range(world)]
+        spread[name] = max(tot) / min(tot)
+    assert spread["work"] < 1.01 and spread["count"] > 1.5

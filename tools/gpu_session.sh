@@ -12,3 +12,7 @@ timeout 900 python bench.py > $O/bench.json 2> $O/bench.err
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/launches.csv python bench.py --steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline --no-direct-count > $O/bench_ncu.log 2>&1
 timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k_eval -c 1 -o $O/k_eval_full python tools/profile_eval.py 5 $NPTS 1 > $O/ncu_full.log 2>&1
 ls -la $O
+# multi-rank functional check of the N>1 bench path (2 ranks on one GPU, gloo) and context lines
+SIAC_DIST_BACKEND=gloo timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29517 bench.py --gpus 2 --steps 2 --warmup 3 --config 4 --e2e-steps 1 --no-cpu-baseline > $O/bench_2rank_gloo_cfg4.json 2> $O/bench_2rank.err
+timeout 900 python bench.py --schedule 6 --steps 3 --no-cpu-baseline --no-direct-count > $O/bench_elem.json 2> $O/bench_elem.err
+ls -la $O
