@@ -203,16 +203,21 @@ def test_counters_agree_between_schedules(siac_mod):
 
 # ------------------------------------------------------------------ edge cases
 
-def test_random_points_anywhere_wrap(siac_mod, oracle_mod):
+EDGE_SCHEDULES = [0, 4, 6]     # default (JUMPX), JUMP, per-element
+
+
+@pytest.mark.parametrize("sch", EDGE_SCHEDULES)
+def test_random_points_anywhere_wrap(siac_mod, oracle_mod, sch):
     """Points outside [0,1)^2 wrap (periodic), including exact corners and edges."""
     w = cfg(2, "random")
     P = np.random.default_rng(1).uniform(-1.5, 2.5, (3000, 2))
     P[:6] = [[0, 0], [1, 1], [1, 0], [0.5, 1.0], [-1e-17, 0.3], [0.999999999999, 0.2]]
-    assert_parity(gpu_eval(siac_mod, w, P), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, P))
+    assert_parity(gpu_eval(siac_mod, w, P, schedule=sch), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, P))
 
 
+@pytest.mark.parametrize("sch", EDGE_SCHEDULES)
 @pytest.mark.parametrize("k", [1, 2, 3, 4])
-def test_structured_breaklines_on_mesh_lines(siac_mod, oracle_mod, k):
+def test_structured_breaklines_on_mesh_lines(siac_mod, oracle_mod, k, sch):
     """h = mesh spacing: kernel breaklines coincide with mesh lines (odd k) or mid-lines
     (even k); points at vertices, edge midpoints and cell centres; random field."""
     N = 16
@@ -224,24 +229,28 @@ def test_structured_breaklines_on_mesh_lines(siac_mod, oracle_mod, k):
     X = np.concatenate([g1, g2])
     P = np.array([[x, y] for x in X[::3] for y in X[::2]])
     ctx = siac_mod.create(V, T, C, k, h)
+    ctx.set_schedule(sch)
     g = ctx.eval(P)
     ctx.destroy()
     assert_parity(g, oracle_mod.oracle_eval(V, T, C, k, h, P))
 
 
-def test_stencil_equals_period(siac_mod, oracle_mod):
+@pytest.mark.parametrize("sch", EDGE_SCHEDULES)
+def test_stencil_equals_period(siac_mod, oracle_mod, sch):
     """W = (3k+1)h = period (k=1, N=4, h=1/4): every triangle meets the stencil through
     several periodic images (SURVEY A4 case)."""
     V, T = inputs.structured_mesh(4)
     C = inputs.random_modes(len(T), 1, seed=2)
     P = np.random.default_rng(3).uniform(0, 1, (200, 2))
     ctx = siac_mod.create(V, T, C, 1, 0.25)
+    ctx.set_schedule(sch)
     g = ctx.eval(P)
     ctx.destroy()
     assert_parity(g, oracle_mod.oracle_eval(V, T, C, 1, 0.25, P))
 
 
-def test_non_periodic_zero_extension(siac_mod, oracle_mod):
+@pytest.mark.parametrize("sch", EDGE_SCHEDULES)
+def test_non_periodic_zero_extension(siac_mod, oracle_mod, sch):
     V, T = inputs.lattice_delaunay_mesh(3000, seed=9)
     k = 2
     C = inputs.random_modes(len(T), k, seed=4)
@@ -249,43 +258,51 @@ def test_non_periodic_zero_extension(siac_mod, oracle_mod):
     P = np.random.default_rng(5).uniform(-0.2, 1.2, (1500, 2))
     for per in (0, 1, 2):
         ctx = siac_mod.create(V, T, C, k, h, periodic=per)
+        ctx.set_schedule(sch)
         g = ctx.eval(P)
         ctx.destroy()
         assert_parity(g, oracle_mod.oracle_eval(V, T, C, k, h, P, periodic=per))
 
 
-def test_graded_small_h_and_large_h(siac_mod, oracle_mod):
-    """h other than the max edge: smaller (triangles span many kernel cells) and larger."""
+@pytest.mark.parametrize("sch", EDGE_SCHEDULES)
+def test_graded_small_h_and_large_h(siac_mod, oracle_mod, sch):
+    """h other than the max edge: smaller (triangles span many kernel cells: the general
+    clip-and-integrate path inside the jump schedules) and larger."""
     V, T = inputs.lattice_delaunay_mesh(2000, seed=12, graded=True)
     C = inputs.random_modes(len(T), 2, seed=6)
     P = inputs.eval_points(V, T, 2)[::17]
     for h in (0.25 * inputs.max_edge(V, T), 0.12):
         ctx = siac_mod.create(V, T, C, 2, h)
+        ctx.set_schedule(sch)
         g = ctx.eval(P)
         ctx.destroy()
         assert_parity(g, oracle_mod.oracle_eval(V, T, C, 2, h, P))
 
 
-def test_single_triangle_and_empty(siac_mod, oracle_mod):
+@pytest.mark.parametrize("sch", EDGE_SCHEDULES)
+def test_single_triangle_and_empty(siac_mod, oracle_mod, sch):
     V = np.array([[0.2, 0.3], [0.45, 0.31], [0.3, 0.5]])
     T = np.array([[0, 1, 2]], dtype=np.int32)
     C = inputs.random_modes(1, 3, seed=1)
     P = np.random.default_rng(2).uniform(0, 1, (257, 2))
     ctx = siac_mod.create(V, T, C, 3, 0.05, periodic=0)
+    ctx.set_schedule(sch)
     assert ctx.eval(np.zeros((0, 2))).shape == (0,)
     g = ctx.eval(P)
     ctx.destroy()
     assert_parity(g, oracle_mod.oracle_eval(V, T, C, 3, 0.05, P, periodic=0))
     ctx0 = siac_mod.create(np.zeros((0, 2)), np.zeros((0, 3), np.int32), np.zeros((0, 3)), 1, 0.1)
+    ctx0.set_schedule(sch)
     assert np.all(ctx0.eval(P) == 0.0)
     ctx0.destroy()
 
 
+@pytest.mark.parametrize("sch", [0, 6])
 @pytest.mark.parametrize("n", [1, 31, 32, 33, 1000, 4097])
-def test_ragged_point_counts(siac_mod, oracle_mod, n):
+def test_ragged_point_counts(siac_mod, oracle_mod, n, sch):
     w = cfg(2, "random")
     P = w.points[sample_idx(w.n_points, n, seed=n)]
-    assert_parity(gpu_eval(siac_mod, w, P), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, P))
+    assert_parity(gpu_eval(siac_mod, w, P, schedule=sch), oracle_mod.oracle_eval(w.V, w.T, w.C, w.k, w.h, P))
 
 
 def test_async_torch_stream(siac_mod, oracle_mod):
