@@ -233,13 +233,20 @@ void eval_device(siac_ctx *c, const double *d_pts, int64_t np, double *d_out, cu
     ensure_scratch(c, np);
     const double Lx = c->dom[2] - c->dom[0], Ly = c->dom[3] - c->dom[1];
     const bool elem = c->schedule == 6;          // per-element: points in row-major cell order
-    k_point_keys<<<nblk(np, 256), 256, 0, st>>>(d_pts, np, c->dom[0], c->dom[1], Lx, Ly, c->periodic, c->cw,
-                                                c->chh, c->ncx, c->ncy, c->d_keys[0], c->d_idx[0], elem ? 1 : 0);
+#ifndef SIAC_TILE_REFINE
+#define SIAC_TILE_REFINE 4
+#endif
+    // point tiles: Morton order of a grid SIAC_TILE_REFINE x finer than the binning cells (more
+    // compact 32-point tiles -> fewer candidates per tile); per-element: row-major binning cells
+    const int rf = elem ? 1 : std::max(1, std::min(SIAC_TILE_REFINE, 65536 / std::max(c->ncx, c->ncy)));
+    k_point_keys<<<nblk(np, 256), 256, 0, st>>>(d_pts, np, c->dom[0], c->dom[1], Lx, Ly, c->periodic, c->cw / rf,
+                                                c->chh / rf, c->ncx * rf, c->ncy * rf, c->d_keys[0], c->d_idx[0],
+                                                elem ? 1 : 0);
     CK(cudaGetLastError());
     cub::DoubleBuffer<uint32_t> kb(c->d_keys[0], c->d_keys[1]);
     cub::DoubleBuffer<int> vb(c->d_idx[0], c->d_idx[1]);
     int end_bit = 1;
-    while ((1ull << end_bit) <= (unsigned long long)std::max(c->ncx, c->ncy) && end_bit < 16) ++end_bit;
+    while ((1ull << end_bit) <= (unsigned long long)std::max(c->ncx, c->ncy) * rf && end_bit < 16) ++end_bit;
     int key_bits = 2 * end_bit;
     if (elem) {
         key_bits = 1;
