@@ -117,6 +117,16 @@ siac_status siac_eval(siac_ctx *ctx, const double *points_xy, int64_t n_points, 
 siac_status siac_eval_async(siac_ctx *ctx, const double *d_points_xy, int64_t n_points,
                             double *d_values_out, void *cuda_stream);
 
+/* CUDA graphs for repeated evaluations (default off).  When enabled, siac_eval_async on a
+ * non-NULL stream captures the whole evaluation (point keys, sort, evaluation kernel) into a
+ * CUDA graph the first time it sees a (d_points_xy, n_points, d_values_out, schedule)
+ * combination and replays it afterwards (up to 8 cached graphs per context, least recently
+ * created evicted first): launch-bound small evaluations cost one graph launch.  The caller
+ * must not free or reallocate those buffers while graphs are enabled; disabling (enable = 0)
+ * drops every cached graph.  Counting, timing and the NULL stream bypass the graphs.  Results
+ * are bitwise those of the direct path. */
+siac_status siac_set_graphs(siac_ctx *ctx, int32_t enable);
+
 /* Evaluation schedule (same result up to rounding):
  *   SIAC_SCHEDULE_DEFAULT (0) the fastest measured schedule (currently SIAC_SCHEDULE_JUMPX);
  *   SIAC_SCHEDULE_POINT   (1) one thread per point, clip and integrate inline (the paper's

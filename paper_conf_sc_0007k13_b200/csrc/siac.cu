@@ -64,6 +64,16 @@ struct siac_ctx {
     bool counting = false;
     unsigned long long *d_cnt = nullptr;
     int64_t last_np = 0;
+    // CUDA graphs of whole evaluations (siac_set_graphs): one per (points, n, values, schedule)
+    bool graphs = false;
+    struct GraphEntry {
+        const double *pts;
+        int64_t np;
+        double *out;
+        int schedule;
+        cudaGraphExec_t exec;
+    };
+    std::vector<GraphEntry> gcache;
     // main-kernel timing (CUDA events on the evaluation stream)
     bool timing = false;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ev;
@@ -203,8 +213,11 @@ __global__ void k_point_keys(const double *pts, int64_t np, double x0, double y0
 
 inline unsigned nblk(int64_t n, int bs) { return (unsigned)((n + bs - 1) / bs); }
 
+void clear_graphs(siac_ctx *c);
+
 void ensure_scratch(siac_ctx *c, int64_t np) {
     if (np <= c->cap) return;
+    clear_graphs(c);                 // captured graphs point at the old scratch buffers
     int64_t cap = std::max<int64_t>(np, c->cap * 3 / 2);
     for (int b = 0; b < 2; ++b) {
         if (c->d_keys[b]) cudaFree(c->d_keys[b]);
@@ -319,9 +332,15 @@ __global__ void __launch_bounds__(512) k_dfma_probe(double *out, int iters, doub
     if (s == 1234.5678) out[blockIdx.x] = s;   // never true; keeps the chains alive
 }
 
+void clear_graphs(siac_ctx *c) {
+    for (auto &g : c->gcache) cudaGraphExecDestroy(g.exec);
+    c->gcache.clear();
+}
+
 void free_ctx(siac_ctx *c) {
     if (!c) return;
     cudaSetDevice(c->device);
+    clear_graphs(c);
     for (auto &e : c->ev) { cudaEventDestroy(e.first); cudaEventDestroy(e.second); }
     void *ptrs[] = {c->d_rec, c->d_jrec, c->d_xrec, c->d_pcell, c->d_bbox, c->d_cell_start, c->d_kc, c->d_keys[0], c->d_keys[1],
                     c->d_idx[0], c->d_idx[1], c->d_cub, c->d_hpts, c->d_hout, c->d_cnt, c->d_tile_counter};
@@ -533,8 +552,54 @@ siac_status siac_eval_async(siac_ctx *ctx, const double *d_pts, int64_t np, doub
         need(np >= 0, "negative n_points");
         if (np == 0) return;
         need(d_pts && d_out, "NULL device pointers");
-        eval_device(ctx, d_pts, np, d_out, (cudaStream_t)stream);
+        cudaStream_t st = (cudaStream_t)stream;
+        if (!ctx->graphs || ctx->counting || ctx->timing || st == nullptr) {
+            eval_device(ctx, d_pts, np, d_out, st);
+            return;
+        }
+        // replay a captured graph of the whole evaluation (keys, sort, kernels) when the same
+        // buffers come back: launch-bound small evaluations pay one graph launch
+        CK(cudaSetDevice(ctx->device));
+        ensure_scratch(ctx, np);
+        if (ctx->schedule == 6 && !ctx->d_pcell)
+            CK(cudaMalloc(&ctx->d_pcell, sizeof(int) * ((int64_t)ctx->ncx * ctx->ncy + 1)));
+        for (auto &g : ctx->gcache)
+            if (g.pts == d_pts && g.np == np && g.out == d_out && g.schedule == ctx->schedule) {
+                CK(cudaGraphLaunch(g.exec, st));
+                return;
+            }
+        if (ctx->gcache.empty()) eval_device(ctx, d_pts, np, d_out, st);   // first use: kernel attributes
+        cudaGraph_t graph = nullptr;
+        CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed));
+        try {
+            eval_device(ctx, d_pts, np, d_out, st);
+        } catch (...) {
+            cudaStreamEndCapture(st, &graph);
+            if (graph) cudaGraphDestroy(graph);
+            throw;
+        }
+        CK(cudaStreamEndCapture(st, &graph));
+        cudaGraphExec_t exec = nullptr;
+        const cudaError_t ie = cudaGraphInstantiate(&exec, graph, 0);
+        cudaGraphDestroy(graph);
+        CK(ie);
+        if (ctx->gcache.size() >= 8) {
+            cudaGraphExecDestroy(ctx->gcache.front().exec);
+            ctx->gcache.erase(ctx->gcache.begin());
+        }
+        ctx->gcache.push_back({d_pts, np, d_out, ctx->schedule, exec});
+        CK(cudaGraphLaunch(exec, st));
     });
+}
+
+siac_status siac_set_graphs(siac_ctx *ctx, int32_t enable) {
+    if (!ctx) { g_err = "NULL context"; return SIAC_EINVAL; }
+    ctx->graphs = enable != 0;
+    if (!ctx->graphs) {
+        cudaSetDevice(ctx->device);
+        clear_graphs(ctx);
+    }
+    return SIAC_OK;
 }
 
 siac_status siac_eval(siac_ctx *ctx, const double *pts, int64_t np, double *out) {

@@ -135,6 +135,8 @@ def lib():
         L.siac_stats.argtypes = [vp, ctypes.POINTER(_Counters)]
         L.siac_set_schedule.restype = ctypes.c_int
         L.siac_set_schedule.argtypes = [vp, I32]
+        L.siac_set_graphs.restype = ctypes.c_int
+        L.siac_set_graphs.argtypes = [vp, I32]
         L.siac_set_timing.restype = ctypes.c_int
         L.siac_set_timing.argtypes = [vp, I32]
         L.siac_timing.restype = ctypes.c_int
@@ -167,7 +169,7 @@ def lib():
 
 
 EXPORTED = ["siac_create", "siac_eval", "siac_eval_async", "siac_set_counting", "siac_stats",
-            "siac_set_schedule", "siac_set_timing", "siac_timing", "siac_probe_fp64",
+            "siac_set_schedule", "siac_set_graphs", "siac_set_timing", "siac_timing", "siac_probe_fp64",
             "siac_info", "siac_host_tables", "siac_debug_records",
             "siac_destroy", "siac_last_error", "siac_version",
             "siac_projection_rule", "siac_map_points_async", "siac_project_async", "siac_error_norms_async"]
@@ -249,6 +251,10 @@ class Context:
         """0 = default (fastest = 5), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump,
         5 = jump with closed-form cross terms, 6 = per-element (the paper's Alg. 3 mapping, scatter-add)."""
         _check(lib().siac_set_schedule(self._ptr, int(schedule)), self._ptr)
+
+    def set_graphs(self, on: bool = True) -> None:
+        """Replay CUDA graphs of repeated eval_async calls on the same buffers (siac_set_graphs)."""
+        _check(lib().siac_set_graphs(self._ptr, 1 if on else 0), self._ptr)
 
     def set_timing(self, on: bool = True) -> None:
         _check(lib().siac_set_timing(self._ptr, 1 if on else 0), self._ptr)
