@@ -123,7 +123,7 @@ __global__ void __launch_bounds__(128) k_eval_v1(EvalArgs a) {
 
 #if SIAC_PART == 0
 template <int K>
-cudaError_t launch_part(const EvalArgs &a, bool count, int *, int, cudaStream_t st) {
+cudaError_t launch_part(const EvalArgs &a, bool count, int *, int num_sms, cudaStream_t st) {
 
     siacjump::JumpArgs j;
     j.pts = a.pts; j.perm = a.perm; j.np = a.np; j.out = a.out; j.rec = a.rec; j.jrec = a.jrec; j.xrec = a.xrec;
@@ -132,7 +132,12 @@ cudaError_t launch_part(const EvalArgs &a, bool count, int *, int, cudaStream_t 
     j.inv_h = a.inv_h; j.hw = a.hw; j.cw = a.cw; j.chh = a.chh; j.ex = a.ex; j.ey = a.ey;
     j.ncx = a.ncx; j.ncy = a.ncy; j.periodic = a.periodic; j.cnt = a.cnt;
     const int64_t ntiles = (a.np + 31) / 32;
-    const unsigned grid = (unsigned)((ntiles + siacjump::WARPS - 1) / siacjump::WARPS);
+    // fewer tiles than ~two waves of resident warps: split each tile's rows over 2 or 4 warps
+    int split = 1;
+    while (split < 4 && split < siacjump::WARPS && ntiles * split < (int64_t)num_sms * 16 * 2) split *= 2;
+    j.split = split;
+    const int tpb = siacjump::WARPS / split;
+    const unsigned grid = (unsigned)((ntiles + tpb - 1) / tpb);
     const size_t smem = ((a.xpoly ? sizeof(siacjump::WarpSmemX) : sizeof(siacjump::WarpSmem)) +
                          sizeof(siacjump::WarpStage<K>)) * siacjump::WARPS;
     // GEN: some triangle is wider than h (in x or y), so a pair may see two knots on an axis
@@ -228,7 +233,7 @@ cudaError_t SIAC_CAT(siac_launch_elem_k, SIAC_K)(const EvalArgs &a, bool count, 
     if (a.nt == 0) return cudaSuccess;
     siacjump::JumpArgs j;
     j.pts = a.pts; j.perm = a.perm; j.np = a.np; j.out = a.out; j.rec = a.rec; j.jrec = a.jrec; j.xrec = a.xrec;
-    j.pcell_start = a.pcell_start; j.bbox = a.bbox; j.cell_start = a.cell_start; j.kc = a.kc;
+    j.pcell_start = a.pcell_start; j.bbox = a.bbox; j.cell_start = a.cell_start; j.kc = a.kc; j.split = 1;
     j.x0 = a.x0; j.y0 = a.y0; j.Lx = a.Lx; j.Ly = a.Ly; j.inv_h = a.inv_h; j.hw = a.hw; j.cw = a.cw; j.chh = a.chh;
     j.ex = a.ex; j.ey = a.ey; j.ncx = a.ncx; j.ncy = a.ncy; j.periodic = a.periodic; j.cnt = a.cnt;
     const unsigned grid = (unsigned)((a.nt + siacjump::WARPS - 1) / siacjump::WARPS);

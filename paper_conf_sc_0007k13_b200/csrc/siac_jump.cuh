@@ -392,6 +392,7 @@ struct JumpArgs {
     const double *jrec;       // JRec<K>
     const double *xrec;       // XRec<K> (closed-form cross terms)
     const int *pcell_start;   // schedule ELEM: CSR of the points sorted by row-major binning cell
+    int split;                // warps per point tile (1, 2, 4): the tile's candidate rows are split
     const double4 *bbox;
     const int *cell_start;
     const double *kc;
@@ -873,8 +874,13 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
     const int wid = threadIdx.x >> 5;
     WS &S = wsm[wid];
     WarpStage<K> &T = reinterpret_cast<WarpStage<K> *>(wsm + WARPS)[wid];
-    const int64_t p0 = ((int64_t)blockIdx.x * WARPS + wid) * 32;
-    if (p0 >= a.np) return;                       // warp-uniform
+    // a.split warps share one tile (small problems: more warps than tiles), each walking a
+    // contiguous share of its candidate rows; partial sums are combined in a fixed order
+    const int split = a.split;
+    const int part = wid % split;
+    const int64_t p0 = ((int64_t)blockIdx.x * (WARPS / split) + wid / split) * 32;
+    const bool live = p0 < a.np;
+    if (split == 1 && !live) return;              // warp-uniform
     if (lane == 0) {
         for (int i = 0; i < NST; ++i) mb_init(&T.bar[i], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -882,7 +888,7 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
     __syncwarp();
     int g = 0;                                    // records streamed so far (ring position)
     unsigned ph = 0;                              // per-slot phase parity
-    const bool valid = p0 + lane < a.np;
+    const bool valid = live && p0 + lane < a.np;
     const int nvalid = __popc(__ballot_sync(0xffffffffu, valid));
     int orig = -1;
     double x1 = 0, x2 = 0;
@@ -908,6 +914,13 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
     int C0 = (int)floor((bx0 - a.ex - a.x0) / a.cw) - 1, C1 = (int)floor((bx1 - a.x0) / a.cw) + 1;
     if (!(a.periodic & 2)) { R0 = max(R0, 0); R1 = min(R1, a.ncy - 1); }
     if (!(a.periodic & 1)) { C0 = max(C0, 0); C1 = min(C1, a.ncx - 1); }
+    if (!live) {
+        R0 = 0; R1 = -1;                          // idle warp of a split block: empty walk
+    } else if (split > 1) {
+        const int nr = R1 - R0 + 1;
+        const int r_lo = R0 + (nr * part) / split, r_hi = R0 + (nr * (part + 1)) / split - 1;
+        R0 = r_lo; R1 = r_hi;
+    }
     __syncwarp();
 
     double acc = 0.0;
@@ -1095,7 +1108,18 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
             }
         });
     }
-    if (valid) a.out[orig] = acc + S.acc[lane];
+    if (split == 1) {
+        if (valid) a.out[orig] = acc + S.acc[lane];
+    } else {
+        __shared__ double psum[WARPS][32];
+        psum[wid][lane] = acc + S.acc[lane];
+        __syncthreads();
+        if (part == 0 && valid) {
+            double t = psum[wid][lane];
+            for (int q = 1; q < split; ++q) t += psum[wid + q][lane];
+            a.out[orig] = t;
+        }
+    }
     if (COUNT) {
         unsigned long long v[8] = {c_cand, c_pairs, c_pieces, c_sub, c_corner, c_cross, c_xsub, c_xpoly};
 #pragma unroll
