@@ -347,7 +347,10 @@ __global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec) {
 #define SIAC_JUMP_PREFETCH 2      // candidates ahead whose hot record lines are prefetched into L1
 #endif
 constexpr int WARPS = SIAC_JUMP_WARPS;
-constexpr int QCAP = 64;      // cross-term queue: < 32 left over + 32 new
+#ifndef SIAC_JUMP_ILP2
+#define SIAC_JUMP_ILP2 0          // 1: two staged records evaluated per step (interleaved arithmetic)
+#endif
+constexpr int QCAP = SIAC_JUMP_ILP2 ? 96 : 64;   // cross-term queue: < 32 left over + 32 (64) new
 constexpr int SCAP = 96;      // staged cross sub-triangles: < 32 left over + <= 64 new
 
 template <int SC> struct WarpSmemT {
@@ -934,7 +937,7 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
     // then body(tri, rsx, rsy, hit, hr) for every candidate whose box meets the tile's stencils
     // (stg = true: only those some lane's stencil meets, hr = the record's hot part in shared
     // memory; else hr = nullptr).
-    auto candidates = [&](auto stg, auto &&body) {
+    auto candidates = [&](auto stg, auto &&body, auto &&body2) {
         for (int R = R0; R <= R1; ++R) {
             int r = R, qy = 0;
             if (a.periodic & 2) { r = ((R % a.ncy) + a.ncy) % a.ncy; qy = (R - r) / a.ncy; }
@@ -985,6 +988,30 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
                                 bulk_load(T.rec[sl], a.jrec + (int64_t)J::RS * (t_cur + T.hj[r]), HB, &T.bar[sl]);
                             }
                         }
+#if SIAC_JUMP_ILP2
+                        for (int i = 0; i < nh; i += 2) {
+                            const bool two = i + 1 < nh;                     // warp-uniform
+                            const int sa = (g + i) & (NST - 1), sb = (g + i + 1) & (NST - 1);
+                            mb_wait(&T.bar[sa], (ph >> sa) & 1u);
+                            ph ^= 1u << sa;
+                            if (two) {
+                                mb_wait(&T.bar[sb], (ph >> sb) & 1u);
+                                ph ^= 1u << sb;
+                            }
+                            const bool ha = ((T.hm[i] >> lane) & 1u) != 0;
+                            const bool hb = two && ((T.hm[i + 1] >> lane) & 1u) != 0;
+                            body2(t_cur + T.hj[i], ha, T.rec[sa], t_cur + T.hj[two ? i + 1 : i], hb,
+                                  T.rec[two ? sb : sa], rsx, rsy);
+                            __syncwarp();
+                            if (lane == 0) {
+                                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                                if (i + NST < nh)
+                                    bulk_load(T.rec[sa], a.jrec + (int64_t)J::RS * (t_cur + T.hj[i + NST]), HB, &T.bar[sa]);
+                                if (i + 1 + NST < nh)
+                                    bulk_load(T.rec[sb], a.jrec + (int64_t)J::RS * (t_cur + T.hj[i + 1 + NST]), HB, &T.bar[sb]);
+                            }
+                        }
+#else
                         for (int i = 0; i < nh; ++i) {
                             const int sl = (g + i) & (NST - 1);
                             mb_wait(&T.bar[sl], (ph >> sl) & 1u);
@@ -996,6 +1023,7 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
                                 bulk_load(T.rec[sl], a.jrec + (int64_t)J::RS * (t_cur + T.hj[i + NST]), HB, &T.bar[sl]);
                             }
                         }
+#endif
                         g += nh;
                     } else {
                         for (int i = 0; i < nk; ++i) {
@@ -1011,10 +1039,13 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
         }
     };
 
-    candidates(std::true_type{}, [&](int tri, double rsx, double rsy, bool hit, const double *hr) {
-        // Every lane evaluates the closed form (no divergence); only lanes whose stencil box
-        // meets the triangle's box add it (and queue its cross term): the four terms of a pair
-        // cancel to rounding only together, so a pair is taken whole or not at all.
+    // One pair = eval (pure arithmetic on the staged record) + commit (accumulate, queue the
+    // cross term).  Every lane evaluates the closed form (no divergence); only lanes whose
+    // stencil box meets the triangle's box add it (and queue its cross term): the four terms of a
+    // pair cancel to rounding only together, so a pair is taken whole or not at all.
+    struct PairV { double v; Cut cx, cy; bool skip; };
+    auto pair_eval = [&](double rsx, double rsy, bool hit, const double *hr) -> PairV {
+        PairV r;
         const double2 cen = ldr2<true>(hr);
         constexpr double MT0 = 0.5 * (3 * K + 1);      // -T0
         const double dx = fma((cen.x + rsx) - x1, a.inv_h, MT0);
@@ -1056,10 +1087,15 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
 #pragma unroll
         for (int j = 0; j <= K; ++j) cc[j] = ux ? q[j] : p[j];
         const double lam = ux ? cx.lam : (uy ? cy.lam : 0.0);
-        v = fma(sg, corner_eval<K, true>(hr + J::OFF_G + sd * J::NGP, cc, lam), v);
-        if (hit && !skip) acc += v;
-        const bool cross = hit && !skip && cx.cut && cy.cut;
-        if (COUNT && hit && !skip) c_corner += (int)cx.cut + (int)cy.cut;
+        r.v = fma(sg, corner_eval<K, true>(hr + J::OFF_G + sd * J::NGP, cc, lam), v);
+        r.cx = cx; r.cy = cy; r.skip = skip;
+        return r;
+    };
+    auto pair_commit = [&](int tri, bool hit, const PairV &r) {
+        const Cut &cx = r.cx, &cy = r.cy;
+        if (hit && !r.skip) acc += r.v;
+        const bool cross = hit && !r.skip && cx.cut && cy.cut;
+        if (COUNT && hit && !r.skip) c_corner += (int)cx.cut + (int)cy.cut;
         const unsigned cm = __ballot_sync(0xffffffffu, cross);
         if (cm) {
             if (cross) {
@@ -1074,16 +1110,32 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
             nq += __popc(cm);
             if (COUNT) c_cross += __popc(cm) * (lane == 0);
             __syncwarp();
-            if (nq >= 32) {
-                if constexpr (XP) {
-                    cross_stage<K, COUNT>(a, S, kcp, alpha, nq, lane, c_xpoly);
-                } else {
-                    clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
-                    while (ns >= 32) integrate_stage<K>(a, S, alpha, ns, lane);
-                }
+        }
+    };
+    auto flush = [&]() {        // integrate queued cross terms 32 at a time (warp-uniform nq)
+        while (nq >= 32) {
+            if constexpr (XP) {
+                cross_stage<K, COUNT>(a, S, kcp, alpha, nq, lane, c_xpoly);
+            } else {
+                clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
+                while (ns >= 32) integrate_stage<K>(a, S, alpha, ns, lane);
             }
         }
-    });
+    };
+    candidates(std::true_type{},
+        [&](int tri, double rsx, double rsy, bool hit, const double *hr) {
+            pair_commit(tri, hit, pair_eval(rsx, rsy, hit, hr));
+            flush();
+        },
+        // two staged records at once (SIAC_JUMP_ILP2): both evaluations are independent
+        // straight-line arithmetic the compiler interleaves; hb = false: B is a dummy (odd tail)
+        [&](int ta, bool ha, const double *ra, int tb, bool hb, const double *rb, double rsx, double rsy) {
+            const PairV va = pair_eval(rsx, rsy, ha, ra);
+            const PairV vb = pair_eval(rsx, rsy, hb, rb);
+            pair_commit(ta, ha, va);
+            pair_commit(tb, hb, vb);
+            flush();
+        });
     if constexpr (XP) {
         while (nq > 0) cross_stage<K, COUNT>(a, S, kcp, alpha, nq, lane, c_xpoly);
     } else {
@@ -1106,7 +1158,7 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
                 acc += go.v;
                 if (COUNT) { c_pieces += go.pieces; c_sub += go.subtris; }
             }
-        });
+        }, 0);
     }
     if (split == 1) {
         if (valid) a.out[orig] = acc + S.acc[lane];
