@@ -347,6 +347,9 @@ __global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec) {
 #define SIAC_JUMP_PREFETCH 2      // candidates ahead whose hot record lines are prefetched into L1
 #endif
 constexpr int WARPS = SIAC_JUMP_WARPS;
+#ifndef SIAC_JUMP_LEAN
+#define SIAC_JUMP_LEAN 1          // 1: paired cell-table loads, one alpha read per pair (default; 0 = previous form)
+#endif
 #ifndef SIAC_JUMP_ILP2
 #define SIAC_JUMP_ILP2 0          // 1: two staged records evaluated per step (interleaved arithmetic)
 #endif
@@ -494,6 +497,15 @@ __device__ __forceinline__ Cut axis_cut(const double *ad, double dd) {
 // zeta.  kcp: padded cell table, row i+1 = cell i, rows 0 and NC+1 zero.
 template <int K>
 __device__ __forceinline__ void base_taylor(const double *kcp, int row, double e, double *p) {
+#if SIAC_JUMP_LEAN
+    if constexpr ((K & 1) == 1) {     // even row length: 16-byte aligned rows, paired loads
+#pragma unroll
+        for (int j = 0; j <= K; j += 2) {
+            const double2 t = *reinterpret_cast<const double2 *>(kcp + row * (K + 1) + j);
+            p[j] = t.x; p[j + 1] = t.y;
+        }
+    } else
+#endif
 #pragma unroll
     for (int j = 0; j <= K; ++j) p[j] = kcp[row * (K + 1) + j];
 #pragma unroll
@@ -860,7 +872,7 @@ template <int K, bool COUNT, bool GEN, bool XP>
 __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_MINB) k_eval_jump(JumpArgs a) {
     using J = JRec<K>;
     constexpr int NC = 3 * K + 1;
-    __shared__ double kcp[(NC + 2) * (K + 1)];
+    __shared__ __align__(16) double kcp[(NC + 2) * (K + 1)];
     __shared__ double alpha[NC + 1];
     extern __shared__ __align__(16) unsigned char jump_dsm[];
     using WS = WarpSmemFor<XP>;
@@ -1080,9 +1092,16 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
         // both cut defers its y corner to the cross-term queue (clip_stage)
         const bool ux = cx.cut;
         const bool uy = !cx.cut && cy.cut;
+#if SIAC_JUMP_LEAN
+        const int sdd = ux ? cx.side : cy.side;
+        const double am = alpha[ux ? cx.m : (uy ? cy.m : 0)];   // uncut: lam = 0 zeroes the corner
+        const int sd = ux ? sdd : 2 + sdd;
+        const double sg = sdd == 0 ? am : -am;
+#else
         const double am = ux ? alpha[cx.m] : (uy ? alpha[cy.m] : 0.0);
         const int sd = ux ? cx.side : 2 + cy.side;
         const double sg = (ux ? cx.side : cy.side) == 0 ? am : -am;
+#endif
         double cc[K + 1];
 #pragma unroll
         for (int j = 0; j <= K; ++j) cc[j] = ux ? q[j] : p[j];
@@ -1200,7 +1219,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_eval_elem(JumpArgs a, int64_t nt
     using J = JRec<K>;
     using X = XRec<K>;
     constexpr int NC = 3 * K + 1;
-    __shared__ double kcp[(NC + 2) * (K + 1)];
+    __shared__ __align__(16) double kcp[(NC + 2) * (K + 1)];
     __shared__ double alpha[NC + 1];
     for (int i = threadIdx.x; i < (NC + 2) * (K + 1); i += blockDim.x) {
         const int row = i / (K + 1);
