@@ -350,6 +350,9 @@ constexpr int WARPS = SIAC_JUMP_WARPS;
 #ifndef SIAC_JUMP_LEAN
 #define SIAC_JUMP_LEAN 1          // 1: paired cell-table loads, one alpha read per pair (default; 0 = previous form)
 #endif
+#ifndef SIAC_JUMP_CSEL
+#define SIAC_JUMP_CSEL 0          // 1: corner coefficients by a third Taylor shift, not selects
+#endif
 #ifndef SIAC_JUMP_ILP2
 #define SIAC_JUMP_ILP2 0          // 1: two staged records evaluated per step (interleaved arithmetic)
 #endif
@@ -1103,8 +1106,14 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
         const double sg = (ux ? cx.side : cy.side) == 0 ? am : -am;
 #endif
         double cc[K + 1];
+#if SIAC_JUMP_CSEL
+        // the other axis' Taylor coefficients, recomputed from selected (row, e) instead of
+        // K+1 double selects between p and q
+        base_taylor<K>(kcp, ux ? cy.row : cx.row, ux ? cy.e : cx.e, cc);
+#else
 #pragma unroll
         for (int j = 0; j <= K; ++j) cc[j] = ux ? q[j] : p[j];
+#endif
         const double lam = ux ? cx.lam : (uy ? cy.lam : 0.0);
         r.v = fma(sg, corner_eval<K, true>(hr + J::OFF_G + sd * J::NGP, cc, lam), v);
         r.cx = cx; r.cy = cy; r.skip = skip;
