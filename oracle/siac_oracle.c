@@ -198,8 +198,9 @@ static void pair_integral(const problem *P, long t, double sx, double sy,
     double lo_x = fmax(xmin, Xb[0]), hi_x = fmin(xmax, Xb[nbr - 1]);
     if (!(lo_x < hi_x)) return;
 
-    /* x-breakpoints: vertices, kernel x-breaklines, edge crossings of kernel y-breaklines */
-    double bx[64];
+    /* x-breakpoints: the 2 ends, <= 3 vertices, <= nbr kernel x-breaklines and <= 3 nbr
+     * crossings of the 3 edges with the nbr kernel y-breaklines */
+    double bx[5 + 4 * (3 * MAXK + 2)];
     int nbx = 0;
     bx[nbx++] = lo_x;
     bx[nbx++] = hi_x;
