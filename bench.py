@@ -129,17 +129,31 @@ def workload_desc(w, cfg):
             "points": "degree-2k symmetric-rule nodes per element"}
 
 
-def cpu_baseline(w, sample_stride, nthreads=0):
-    """The oracle as it stands, on a deterministic stride sample of the workload's points,
-    on all host cores (explicit: torchrun sets OMP_NUM_THREADS=1)."""
+def parity_report(g, o, tol=1e-10):
+    """The parity rule of tests/test_gpu_parity.py on one sample: normwise
+    max|g-o|/max|o| and pointwise |g-o|/|o| where |o| >= 1e-2 max|o|."""
+    g, o = np.asarray(g, dtype=np.float64), np.asarray(o, dtype=np.float64)
+    scale = max(float(np.abs(o).max()), 1e-300)
+    err = np.abs(g - o)
+    big = np.abs(o) >= 1e-2 * scale
+    rel = err[big] / np.abs(o[big]) if big.any() else np.zeros(1)
+    nw, pw = float(err.max() / scale), float(rel.max())
+    return {"max_normwise": nw, "max_pointwise": pw, "p99_pointwise": float(np.quantile(rel, 0.99)),
+            "n_points": int(len(o)), "tolerance": tol, "pass": bool(nw <= tol and pw <= tol and np.all(np.isfinite(g)))}
+
+
+def cpu_baseline(w, idx, label, nthreads=0):
+    """The oracle as it stands, on a deterministic sample `idx` of the workload's points, on
+    all host cores (explicit: torchrun sets OMP_NUM_THREADS=1).  Returns the baseline record
+    and the oracle's values at the sample (the bench line's parity check)."""
     import oracle
     nthreads = nthreads or oracle.omp_threads()
-    P = w.points[::sample_stride]
+    P = w.points[idx]
     t0 = time.perf_counter()
-    oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P, nthreads=nthreads)
+    vals = oracle.oracle_eval(w.V, w.T, w.C, w.k, w.h, P, nthreads=nthreads)
     dt = time.perf_counter() - t0
-    return {"value": len(P) / dt, "unit": "points/s", "cores": nthreads or oracle.omp_threads(), "kind": "oracle",
-            "sample": f"every {sample_stride}th evaluation point ({len(P)} points), {dt:.1f} s"}
+    return ({"value": len(P) / dt, "unit": "points/s", "cores": nthreads, "kind": "oracle",
+             "sample": f"{label} ({len(P)} points), {dt:.1f} s"}, vals)
 
 
 def run_reference(args):
@@ -171,6 +185,44 @@ def run_reference(args):
     return 0
 
 
+def broadcast_workload(w, rank, device):
+    """Rank 0's workload (mesh, modes, points) to every rank: the metadata by
+    broadcast_object_list, the arrays by one broadcast each over the process group (NCCL over
+    NVLink on a GPU box).  Returns (workload, broadcast ms of the arrays)."""
+    import types
+
+    import torch
+    import torch.distributed as dist
+
+    meta = [None]
+    if rank == 0:
+        meta = [{"k": w.k, "h": w.h, "seed": w.seed, "name": w.name, "meta": w.meta, "periodic": w.periodic,
+                 "domain": w.domain, "shapes": {n: getattr(w, n).shape for n in ("V", "T", "C", "points")},
+                 "dtypes": {n: str(getattr(w, n).dtype) for n in ("V", "T", "C", "points")}}]
+    dist.broadcast_object_list(meta, src=0, device=device if device.type == "cuda" else None)
+    m = meta[0]
+    if device.type == "cuda":
+        torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    arrs = {}
+    for n in ("V", "T", "C", "points"):
+        dt = {"float64": torch.float64, "int32": torch.int32}[m["dtypes"][n]]
+        if rank == 0:
+            t = torch.from_numpy(np.ascontiguousarray(getattr(w, n))).to(device)
+        else:
+            t = torch.empty(m["shapes"][n], dtype=dt, device=device)
+        dist.broadcast(t, src=0)
+        arrs[n] = t
+    out = {n: t.cpu().numpy() for n, t in arrs.items()}
+    ms = 1e3 * (time.perf_counter() - t0)
+    if rank == 0:
+        return w, ms
+    ns = types.SimpleNamespace(k=m["k"], h=m["h"], seed=m["seed"], name=m["name"], meta=m["meta"],
+                               periodic=m["periodic"], domain=m["domain"], **out)
+    ns.n_points = len(ns.points)
+    return ns, ms
+
+
 def run_siac(args):
     import torch
     import torch.distributed as dist
@@ -184,6 +236,11 @@ def run_siac(args):
     dev = torch.device("cuda", local % max(ndev, 1))
     torch.cuda.set_device(dev)
     backend = os.environ.get("SIAC_DIST_BACKEND", "nccl")     # gloo: functional runs with >1 rank per GPU
+    if world > 1 and backend == "nccl":
+        # NCCL's communicator lines (ranks, NVLink/NVLS transport) go to stderr, not the JSON stdout
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
     if world > 1:
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=dev)
@@ -204,8 +261,21 @@ def run_siac(args):
         dist.all_reduce(t)
         return [int(x) for x in t.tolist()]
 
-    w = load_workload(args.config)
+    def allgather_floats(vals):
+        t = torch.tensor(vals, dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
+        out = torch.empty(world * len(vals), dtype=torch.float64, device=t.device)
+        dist.all_gather_into_tensor(out, t)
+        return out.view(world, len(vals)).tolist()
+
+    # inputs: generated once on rank 0 and broadcast to the other ranks
+    t_in = time.perf_counter()
+    w = load_workload(args.config) if rank == 0 else None
+    bcast_ms = None
+    if world > 1:
+        w, bcast_ms = broadcast_workload(w, rank, dev if backend == "nccl" else torch.device("cpu"))
+    t_in = time.perf_counter() - t_in
     k = w.k
+    halo_info = None
     if world > 1:
         from paper_conf_sc_0007k13_b200 import dist as sdist
         wts = sdist.work_estimate(w.V, w.T, w.points, 0.5 * (3 * k + 1) * w.h)
@@ -215,8 +285,18 @@ def run_siac(args):
     else:
         part = None
         V, T, C, P_local = w.V, w.T, w.C, w.points
+    t0 = time.perf_counter()
     ctx = siac.create(V, T, C, k, w.h, periodic=3, device=dev.index)
+    create_wall_ms = 1e3 * (time.perf_counter() - t0)
+    cinfo = ctx.create_info()
     ctx.set_schedule(args.schedule)
+    if world > 1:
+        per_rank = allgather_floats([float(len(P_local)), float(len(T)), create_wall_ms, cinfo["cross_ms"]])
+        halo_info = {"points": [int(r[0]) for r in per_rank], "halo_triangles": [int(r[1]) for r in per_rank],
+                     "create_ms": [round(r[2], 2) for r in per_rank],
+                     "create_cross_ms": [round(r[3], 2) for r in per_rank],
+                     "mesh_triangles": int(len(w.T)),
+                     "input_broadcast_ms": bcast_ms}
     n_local = len(P_local)
     d_pts = torch.from_numpy(np.ascontiguousarray(P_local)).to(dev)
     d_out = torch.empty(max(n_local, 1), dtype=torch.float64, device=dev)
@@ -264,8 +344,7 @@ def run_siac(args):
             dist.all_gather_into_tensor(gathered, send)
 
     # L2: flush between timed steps unless this rank's inputs alone exceed the 126 MB L2
-    rs = (16 + (k + 1) * (k + 2) // 2 + 1) & ~1
-    in_bytes = n_local * 16 + len(T) * rs * 8
+    in_bytes = n_local * 16 + len(T) * cinfo["bytes_per_triangle"]
     flush = in_bytes < 2 * 126e6
     scrub = torch.empty(int(256e6) // 4, dtype=torch.float32, device=dev) if flush else None
 
@@ -301,12 +380,18 @@ def run_siac(args):
     ms_step = ms_total / args.steps
     value = w.n_points / (ms_step * 1e-3)
 
+    # the values of the last timed step, for the parity check (N > 1: assembled from the gather)
+    vals_local = d_out[:n_local].cpu().numpy()
+    vals_full = None
+    if world > 1 and rank == 0:
+        vals_full = sdist.assemble(gathered.cpu().numpy(), part, w.n_points)
+
     # end-to-end through the public host-buffer API (siac_eval): every step copies this rank's
     # points from pinned host memory, evaluates, copies the values back, and (N > 1) gathers
     # all ranks' values so every rank holds the full result
     h_pts = torch.from_numpy(np.ascontiguousarray(P_local)).pin_memory()
     h_out = torch.empty(max(n_local, 1), dtype=torch.float64).pin_memory()
-    hp, ho = h_pts.numpy(), h_out.numpy()
+    hp, ho = h_pts.numpy().reshape(-1, 2), h_out.numpy()
     ctx.eval_into(hp, ho)
     if world > 1:
         gather(h_out.to(gathered.device))
@@ -320,6 +405,28 @@ def run_siac(args):
             full = gathered.cpu()
     e2e_s = allreduce_max([time.perf_counter() - t0])[0]
     e2e_val = w.n_points / (e2e_s / args.e2e_steps) if args.e2e_steps > 0 else None
+    ctx.destroy()
+
+    # one-shot use (the paper's: one evaluation at the end of a run):
+    # siac_create from host arrays + siac_eval (host buffers) + siac_destroy, per rank, then the
+    # gather; max over ranks
+    oneshot = None
+    if args.oneshot:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        c1 = siac.create(V, T, C, k, w.h, periodic=3, device=dev.index)
+        c1.set_schedule(args.schedule)
+        c1.eval_into(hp, ho)
+        c1.destroy()
+        if world > 1:
+            gather(h_out.to(gathered.device, non_blocking=False))
+            full = gathered.cpu()
+        os_s = allreduce_max([time.perf_counter() - t0])[0]
+        oneshot = {"ms": 1e3 * os_s, "value": w.n_points / os_s, "unit": "points/s",
+                   "note": "siac_create (host arrays) + siac_eval (host buffers) + siac_destroy"
+                           + (" + all_gather, max over ranks" if world > 1 else "")}
 
     peak_meas = siac.probe_fp64(dev.index)
     line = None
@@ -328,18 +435,22 @@ def run_siac(args):
         # whole-job algorithmic flops per launch-set / slowest rank's kernel time / ranks
         achieved = flops_step / world / kern_avg_s / 1e12 if kern_avg_s > 0 else None
         peak = fp64_peak_derived()
-        # DRAM traffic per launch: bytes/point of the committed ncu --set full capture of this
-        # kernel (profiles/r01_ncu_traffic_jumpx.json, a 2M-point subset) x this launch's points
-        traffic = None
-        tpath = os.path.join(ROOT, "profiles", "r01_ncu_traffic_jumpx.json")
-        if args.schedule in (0, 5) and os.path.exists(tpath):
-            traffic = json.load(open(tpath))["bytes_per_point"] * n_local
+        # DRAM traffic per launch from the committed ncu --set full capture of this kernel at
+        # the bench's own cfg-5 launch (profiles/*_ncu_traffic_cfg5.json), scaled by points
+        traffic, ncu_rec = None, None
+        for tp in ("r02_ncu_traffic_cfg5.json", "r01_ncu_traffic_jumpx.json"):
+            tpath = os.path.join(ROOT, "profiles", tp)
+            if args.schedule in (0, 5) and os.path.exists(tpath):
+                ncu_rec = json.load(open(tpath))
+                ncu_rec["file"] = "profiles/" + tp
+                traffic = ncu_rec["bytes_per_point"] * n_local
+                break
         cfgd = workload_desc(w, args.config)
         cfgd.update({"parallelism": f"spatial point tiles x{world} + halo, NCCL all_gather" if world > 1
                      else "single GPU",
                      "l2": ("L2 flushed (256 MB write) between timed steps" if flush else
                             "inputs larger than L2 (points %.0f MB + triangle records %.0f MB > 126 MB)"
-                            % (n_local * 16 / 1e6, len(T) * rs * 8 / 1e6)),
+                            % (n_local * 16 / 1e6, len(T) * cinfo["bytes_per_triangle"] / 1e6)),
                      "counts": {"candidates": cands, "pairs": pairs, "pieces": pieces, "subtris": subtris,
                                 "corner_terms": corners, "cross_terms": crosses, "cross_subtris": xsub,
                                 "cross_polys": xpoly},
@@ -351,32 +462,66 @@ def run_siac(args):
                 "data": "synthetic", "config": cfgd,
                 "roofline": {"bound": "alu", "kernel": "k_eval", "achieved": achieved, "peak": peak,
                              "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,
-                             "traffic_note": "dram read+write bytes per launch, scaled from the committed ncu capture "
-                                             "(profiles/r01_ncu_traffic_jumpx.json); algorithmic ~41 B/point",
-                             "peak_note": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1965 MHz (DESIGN.md)",
+                             "traffic_note": ("dram read+write bytes per launch from the committed ncu --set full "
+                                              "capture (%s), scaled by this launch's points; algorithmic ~41 B/point"
+                                              % (ncu_rec["file"] if ncu_rec else "none")),
+                             "peak_note": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1965 MHz (DESIGN.md §8.1)",
                              "measured_dfma_peak": peak_meas,
                              "frac_of_measured": (achieved / peak_meas) if achieved else None,
                              "kernel_share_of_step": (kern_ms / kern_n) / ms_step if kern_n else None,
                              "algorithmic_flops_per_step": flops_step,
-                             "flop_model": ("JUMP decomposition (DESIGN.md §8.2)" if jump else
+                             "flop_model": ("headline: the JUMP decomposition's own operation count (DESIGN.md "
+                                            "§8.2); see direct_method for SURVEY §8(d)'s per-quadrature-point model "
+                                            "and ncu_executed for the executed FP64 instructions" if jump else
                                             "direct SH + fan + quadrature (SURVEY §8(d))")},
+                "create": {"wall_ms": create_wall_ms, **{k_: cinfo[k_] for k_ in
+                           ("host_ms", "h2d_ms", "index_ms", "jump_ms", "cross_ms", "device_bytes",
+                            "bytes_per_triangle")},
+                           "cross_share_of_eval_step": cinfo["cross_ms"] / ms_step,
+                           "note": "siac_create once per mesh, excluded from value (SURVEY §8(d)); rank 0's"},
                 "e2e": {"value": e2e_val, "unit": "points/s", "h2d_bytes_per_step": int(w.n_points * 16),
                         "d2h_bytes_per_step": int(w.n_points * 8)},
+                "oneshot": oneshot,
                 "schedule": ["default(jump-x)", "point", "tile", "ws", "jump", "jump-x", "elem"][args.schedule],
                 "gpu_launches": 2 * args.steps,
                 "gpu_launches_note": "per step and rank: k_point_keys + k_eval (ours) + CUB radix-sort kernels",
                 "clocks": clk}
+        if ncu_rec is not None and ncu_rec.get("fp64_executed_tflops_equiv") is not None:
+            line["roofline"]["ncu_executed"] = {
+                "fp64_pipe_pct": ncu_rec.get("fp64_pipe_pct"),
+                "executed_frac": ncu_rec.get("fp64_executed_frac"),
+                "note": "(2 DFMA + DADD + DMUL) thread instructions / kernel time / derived peak, ncu capture"}
+        if halo_info is not None:
+            line["multi_gpu"] = halo_info
         if direct is not None:
             dm = direct["model_flops_per_step"]
             direct["model_tflops_equivalent"] = dm / world / kern_avg_s / 1e12 if kern_avg_s > 0 else None
+            direct["model_frac"] = direct["model_tflops_equivalent"] / peak if kern_avg_s > 0 else None
             direct["note"] = ("SURVEY §8(d) model flops of the direct decomposition of the same integral / this "
                               "kernel's time: the work the jump decomposition avoids, not executed flops")
             line["direct_method"] = direct
     if rank == 0 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(w, max(1, w.n_points // args.ref_points))
+        if world == 1:
+            # the oracle timed on a stride sample, and the GPU's values at the same points
+            stride = max(1, w.n_points // args.ref_points)
+            idx = np.arange(0, w.n_points, stride)
+            cb, ovals = cpu_baseline(w, idx, f"every {stride}th evaluation point")
+            line["cpu_baseline"] = cb
+            line["parity"] = dict(parity_report(vals_local[idx], ovals), sample=cb["sample"])
+        else:
+            # N > 1: the assembled (gathered) values against the oracle on points next to the
+            # partition cuts (their values depend on the halos) plus a stride sample
+            hw = 0.5 * (3 * k + 1) * w.h
+            near = sdist.near_cut_points(w.points, part, hw)
+            rng = np.random.default_rng(77)
+            pick = np.sort(rng.choice(near, size=min(len(near), args.ref_points // 4), replace=False))
+            idx = np.unique(np.concatenate([pick, np.arange(0, w.n_points, max(1, 4 * w.n_points // args.ref_points))]))
+            _, ovals = cpu_baseline(w, idx, "near-cut + stride")
+            line["parity"] = dict(parity_report(vals_full[idx], ovals),
+                                  sample=f"{len(pick)} points within W/2 of the {world}-way partition cuts + a stride "
+                                         f"sample, gathered values")
     if rank == 0:
         print(json.dumps(line), flush=True)
-    ctx.destroy()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
@@ -396,6 +541,8 @@ def main():
                     help="0 = default (jump-x), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, "
                          "4 = jump, 5 = jump with closed-form cross terms, 6 = per-element (scatter)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-oneshot", dest="oneshot", action="store_false",
+                    help="skip the one-shot create + eval + destroy timing")
     ap.add_argument("--no-direct-count", dest="direct_count", action="store_false",
                     help="skip the (untimed) direct-decomposition count run")
     args = ap.parse_args()

@@ -50,14 +50,37 @@ typedef enum {
 #define SIAC_PERIODIC_X 1
 #define SIAC_PERIODIC_Y 2
 
+/* Modal basis of the coefficients siac_create reads ("an array of the
+ * polynomial modes"; the basis is not named). */
+typedef enum {
+    SIAC_BASIS_DUBINER_ORTHONORMAL = 0,  /* default; see siac_create */
+    SIAC_BASIS_MONOMIAL_REF = 1          /* u = sum c_i r^a s^b on the unit reference triangle
+                                            (point = v0 + r (v1 - v0) + s (v2 - v0)); mode i
+                                            ordered like the Dubiner modes: by n = a + b, then b */
+} siac_basis;
+
+/* What the stencil does on a NON-periodic axis near the domain boundary (PAPER.md L280-283:
+ * "the stencil either wraps around the domain for periodic solutions, or an asymmetric
+ * (one-sided) stencil is used [21]").  Periodic axes always wrap. */
+typedef enum {
+    SIAC_BOUNDARY_ZERO = 0,      /* symmetric kernel everywhere, u_h = 0 outside the mesh */
+    SIAC_BOUNDARY_ONESIDED = 1   /* position-dependent one-sided kernel (ref [21], Ryan & Shu
+                                    2003; reading R4): the 2k+1 B-spline nodes are
+                                    shifted by lambda(x) so the support stays inside
+                                    [x0, x1] x [y0, y1], and the coefficients c_g(lambda)
+                                    re-solve the same moment conditions (degree-2k
+                                    reproduction); needs W = (3k+1)h <= the extent */
+} siac_boundary;
+
 typedef struct {
     int32_t k;          /* dG degree = B-spline degree; 1..4 (paper tested 1..3, L716-718) */
     double  h;          /* kernel scaling > 0; the paper uses the longest edge s (L430, L440) */
-    int32_t periodic;   /* SIAC_PERIODIC_X | SIAC_PERIODIC_Y; non-periodic axes use zero
-                           extension outside the mesh */
+    int32_t periodic;   /* SIAC_PERIODIC_X | SIAC_PERIODIC_Y; non-periodic axes: see boundary */
     double  domain[4];  /* x0, y0, x1, y1; the paper uses [0,1]^2 (L428) */
     int32_t device;     /* CUDA device ordinal */
     double  cell_factor;/* binning cell size / h; 0 -> default 0.5 (paper c_e = s/2, L505-508) */
+    int32_t basis;      /* siac_basis of `coeffs` (0 = orthonormal Dubiner) */
+    int32_t boundary;   /* siac_boundary for the non-periodic axes (0 = zero extension) */
 } siac_params;
 
 typedef struct {        /* geometry counts of the last evaluation (see siac_set_counting) */
@@ -79,7 +102,8 @@ typedef struct {        /* geometry counts of the last evaluation (see siac_set_
  *   vertices_xy  host, n_vertices x 2 doubles, row-major (x, y).  On periodic axes every
  *                vertex must lie in [x0, x1] (tolerance 1e-9 of the extent).
  *   triangles    host, n_triangles x 3 int32, 0-based vertex indices; any orientation.
- *   coeffs       host, n_triangles x (k+1)(k+2)/2 doubles: coefficients of the orthonormal
+ *   coeffs       host, n_triangles x (k+1)(k+2)/2 doubles: modal coefficients in
+ *                params->basis; default: the orthonormal
  *                Dubiner basis on the reference triangle {xi, eta >= -1, xi + eta <= 0},
  *                triangle vertices 0, 1, 2 mapped to (-1,-1), (1,-1), (-1,1);
  *                phi_pq = sqrt((2p+1)(p+q+1)/2) P_p(a) ((1-eta)/2)^p P_q^(2p+1,0)(eta),
@@ -88,7 +112,8 @@ typedef struct {        /* geometry counts of the last evaluation (see siac_set_
  *   params       see siac_params.
  *   *out         receives the context (NULL on failure).
  * Errors: SIAC_EINVAL for k outside 1..4, h <= 0 or non-finite, (3k+1)h larger than a
- *   periodic extent, an empty or inverted domain, out-of-range indices, zero-area triangles,
+ *   periodic extent (or, with SIAC_BOUNDARY_ONESIDED, than a non-periodic extent), an unknown
+ *   basis or boundary, an empty or inverted domain, out-of-range indices, zero-area triangles,
  *   non-finite coordinates or coefficients, vertices outside a periodic axis; SIAC_EDEVICE,
  *   SIAC_ENOMEM, SIAC_ECUDA.  n_triangles == 0 is allowed (every value is then 0).
  */
@@ -101,8 +126,10 @@ siac_status siac_create(siac_ctx **out,
  * siac_eval -- blocking evaluation with HOST buffers.
  *   points_xy   host, n_points x 2 doubles (x, y); any location (periodic axes wrap).
  *   values_out  host, n_points doubles, written in input order.
- * Includes the host->device copy of the points and the device->host copy of the values.
- * n_points == 0 is a no-op returning SIAC_OK.
+ * Includes the host->device copy of the points and the device->host copy of the values, all
+ * stream-ordered on the context's own stream (pinned host buffers copy at full PCIe rate;
+ * the copies cannot overlap the kernel: the point sort needs every point and the values are
+ * written in input order).  n_points == 0 is a no-op returning SIAC_OK.
  */
 siac_status siac_eval(siac_ctx *ctx, const double *points_xy, int64_t n_points, double *values_out);
 
@@ -200,7 +227,22 @@ siac_status siac_error_norms_async(const double *d_u, const double *d_ref, const
                                    double *d_out, void *cuda_stream);
 
 /* Counters of the last evaluation run with counting enabled (synchronises the device). */
-siac_status siac_stats(siac_ctx *ctx, siac_counters *out);
+siac_status siac_stats(const siac_ctx *ctx, siac_counters *out);
+
+/* Cost and footprint of siac_create (create is excluded from points/s and
+ * "reported separately"; the element data are built once and reused by every evaluation,
+ * PAPER.md L586-594).  Device times are CUDA-event times on the context's stream. */
+typedef struct {
+    double  total_ms;        /* wall clock of siac_create (host + device, until synchronised) */
+    double  host_ms;         /* host validation pass + exact constants */
+    double  h2d_ms;          /* vertices, triangles and modes host -> device */
+    double  index_ms;        /* k_prep + CUB sort by anchor cell + k_gather + k_cell_start */
+    double  jump_ms;         /* k_prep_jump: per-triangle moments and corner polynomials */
+    double  cross_ms;        /* k_prep_cross: interval polynomials of the clipped corners */
+    int64_t device_bytes;    /* device memory the context keeps after siac_create */
+    int64_t bytes_per_triangle;  /* resident per-triangle data (records + box) */
+} siac_create_info;
+siac_status siac_get_create_info(const siac_ctx *ctx, siac_create_info *out);
 
 /* Enable (1) / disable (0) CUDA-event timing of the main evaluation kernel (k_eval) on the
  * evaluation stream.  While enabled, every evaluation records one event pair around it. */

@@ -148,7 +148,7 @@ def gl_sizes(k: int, field_mode: int = 0, field_deg: int = 0) -> tuple[int, int]
       dG field (degree k):      x-degree K1 k + K2 k + u k + Jacobian 1 = 3k+1, eta-degree 2k;
       monomial field y1^i y2^j (i, j <= d): x-degree 2k + 2d + 1, eta-degree k + d.
     An n-point Gauss-Legendre rule is exact to degree 2n-1."""
-    if field_mode == 0:
+    if field_mode in (0, 2):
         dx, dy = 3 * k + 1, 2 * k
     else:
         dx, dy = 2 * k + 2 * field_deg + 1, k + field_deg
@@ -160,8 +160,10 @@ def oracle_eval(V, T, C, k: int, h: float, points, periodic: int = 3,
                 use_grid: bool | None = None, nthreads: int = 0, return_area: bool = False):
     """u*(x) at every point (Eq. (1)); see siac_oracle.c for the method.
 
-    V (nv,2) f64; T (nt,3) int; C: (nt, (k+1)(k+2)/2) Dubiner modes (field_mode 0) or the
-    (d+1)^2 coefficients a[i, j] of y1^i y2^j (field_mode 1, d = field_deg)."""
+    V (nv,2) f64; T (nt,3) int; C: (nt, (k+1)(k+2)/2) Dubiner modes (field_mode 0), the
+    (d+1)^2 coefficients a[i, j] of y1^i y2^j (field_mode 1, d = field_deg), or (field_mode 2,
+    the library's SIAC_BASIS_MONOMIAL_REF) per-triangle coefficients of r^a s^b on the unit
+    reference triangle (y = v0 + r (v1 - v0) + s (v2 - v0)), ordered by a + b, then b."""
     lib = _load()
     V = np.ascontiguousarray(V, dtype=np.float64)
     T = np.ascontiguousarray(T, dtype=np.int32)

@@ -128,7 +128,9 @@ typedef struct {
     const double *V;             /* nv x 2 */
     const int *T;                /* nt x 3 */
     long nt;
-    int field_mode;              /* 0: dG Dubiner modes (nt x nb); 1: global polynomial */
+    int field_mode;              /* 0: dG Dubiner modes (nt x nb); 1: global polynomial;
+                                    2: per-triangle monomials r^a s^b of the unit reference
+                                       triangle (nt x nb, ordered by a+b, then b) */
     const double *field;
     int field_deg;               /* mode 1: coefficients a[i*(deg+1)+j] of y1^i y2^j */
     int nx, ny;                  /* Gauss-Legendre sizes in x and along the strip */
@@ -157,8 +159,14 @@ static double field_value(const problem *P, long t, double y1, double y2)
     double r = (a22 * d1 - a12 * d2) / det;
     double s = (-a21 * d1 + a11 * d2) / det;
     double phi[MAXB];
-    oracle_dubiner(P->k, 2.0 * r - 1.0, 2.0 * s - 1.0, phi);
     int nb = (P->k + 1) * (P->k + 2) / 2;
+    if (P->field_mode == 2) {            /* phi_i = r^(n-b) s^b, i by n = a+b then b */
+        int i = 0;
+        for (int n = 0; n <= P->k; ++n)
+            for (int b = 0; b <= n; ++b) phi[i++] = pow(r, n - b) * pow(s, b);
+    } else {
+        oracle_dubiner(P->k, 2.0 * r - 1.0, 2.0 * s - 1.0, phi);
+    }
     const double *c = P->field + (long)nb * t;
     double u = 0.0;
     for (int i = 0; i < nb; ++i) u += c[i] * phi[i];

@@ -4,13 +4,17 @@
 //   siac_create:  host validation + exact constants (siac_math.hpp) -> H2D of V, T, C ->
 //                 k_prep (per-triangle record, bbox, anchor cell) -> CUB radix sort by anchor
 //                 cell -> k_gather (records in cell order) -> k_cell_start (CSR offsets).
-//   siac_eval_async: k_point_keys (periodic wrap, Morton key of the binning cell) -> CUB
-//                 radix sort -> k_eval (points in Morton order; candidate triangles from the
-//                 cells of the stencil's Eq. (3)-style bounds; per pair: clip, fan, quadrature;
-//                 one accumulator per point, written in input order).
+//                 -> k_prep_jump (moments, corner polynomials) -> k_prep_cross (interval
+//                 polynomials of the clipped reference corners), all on the context's stream.
+//   siac_eval_async: k_point_keys (periodic wrap, Morton key of a grid finer than the binning
+//                 cells) -> CUB radix sort -> the schedule's evaluation kernel (default
+//                 k_eval_jump<K,..,JUMPX>: candidate triangles from the cells of each 32-point
+//                 tile's Eq. (3)-style bounds, the spline-jump decomposition of Eq. (2) in closed
+//                 form per pair, one accumulator per point, written in input order).
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -32,7 +36,10 @@ using namespace siacdev;
 
 struct siac_ctx {
     int device = 0;
+    cudaStream_t stream = nullptr;   // the context's own non-blocking stream (create, siac_eval)
     int k = 1;
+    int basis = 0, boundary = 0;
+    siac_create_info cinfo = {};
     double h = 0, inv_h = 0;
     int periodic = 0;
     double dom[4] = {0, 0, 1, 1};
@@ -56,6 +63,7 @@ struct siac_ctx {
     void *d_cub = nullptr;
     size_t cub_bytes = 0;
     int64_t cap_host = 0;
+    int64_t scratch_bytes = 0;
     double *d_hpts = nullptr, *d_hout = nullptr;
     // counters
     int schedule = 0;            // 0 = default (= 5), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump, 5 = jump-x, 6 = per-element
@@ -346,6 +354,7 @@ void free_ctx(siac_ctx *c) {
                     c->d_idx[0], c->d_idx[1], c->d_cub, c->d_hpts, c->d_hout, c->d_cnt, c->d_tile_counter};
     for (void *p : ptrs)
         if (p) cudaFree(p);
+    if (c->stream) cudaStreamDestroy(c->stream);
     delete c;
 }
 
@@ -381,6 +390,10 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
                         const double *C, const siac_params *p) {
     if (out) *out = nullptr;
     siac_ctx *c = nullptr;
+    const auto t_start = std::chrono::steady_clock::now();
+    auto ms_since = [](std::chrono::steady_clock::time_point t0) {
+        return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    };
     siac_status st = run_guarded(&g_err, [&]() {
         need(out != nullptr && p != nullptr, "out and params must be non-NULL");
         need(p->k >= 1 && p->k <= 4, "k must be in 1..4");
@@ -388,6 +401,8 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
         need(nv >= 0 && nt >= 0, "negative sizes");
         need(nt == 0 || (V && T && C), "NULL mesh arrays");
         need((p->periodic & ~3) == 0, "periodic must be a combination of SIAC_PERIODIC_X|Y");
+        need(p->basis == SIAC_BASIS_DUBINER_ORTHONORMAL || p->basis == SIAC_BASIS_MONOMIAL_REF, "unknown basis");
+        need(p->boundary == SIAC_BOUNDARY_ZERO || p->boundary == SIAC_BOUNDARY_ONESIDED, "unknown boundary");
         for (int i = 0; i < 4; ++i) need(std::isfinite(p->domain[i]), "non-finite domain");
         const double Lx = p->domain[2] - p->domain[0], Ly = p->domain[3] - p->domain[1];
         need(Lx > 0 && Ly > 0, "empty or inverted domain");
@@ -395,6 +410,11 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
         const double W = (3 * k + 1) * p->h;
         need(!(p->periodic & 1) || W <= Lx * (1 + 1e-12), "(3k+1)h exceeds the periodic x-extent");
         need(!(p->periodic & 2) || W <= Ly * (1 + 1e-12), "(3k+1)h exceeds the periodic y-extent");
+        if (p->boundary == SIAC_BOUNDARY_ONESIDED) {
+            need((p->periodic & 1) || W <= Lx * (1 + 1e-12), "one-sided kernel: (3k+1)h exceeds the x-extent");
+            need((p->periodic & 2) || W <= Ly * (1 + 1e-12), "one-sided kernel: (3k+1)h exceeds the y-extent");
+            need(p->periodic == 3, "SIAC_BOUNDARY_ONESIDED is not implemented yet");
+        }
         need(nt <= (int64_t)0x3fffffff, "too many triangles");
         const int nb = (k + 1) * (k + 2) / 2;
         // host validation pass
@@ -429,6 +449,9 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
 
         c = new siac_ctx();
         c->device = p->device;
+        CK(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
+        c->basis = p->basis;
+        c->boundary = p->boundary;
         c->k = k;
         c->h = p->h;
         c->inv_h = 1.0 / p->h;
@@ -444,17 +467,26 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
         c->chh = Ly / c->ncy;
         // exact constants
         std::vector<double> kc = siac::kernel_cell_table(k);
-        std::vector<double> R = siac::dubiner_to_centred(k);
+        std::vector<double> R = p->basis == SIAC_BASIS_MONOMIAL_REF ? siac::monomial_to_centred(k)
+                                                                    : siac::dubiner_to_centred(k);
+        c->cinfo.host_ms = ms_since(t_start);
+        cudaStream_t cs = c->stream;
+        cudaEvent_t ev[5] = {};
+        for (auto &e : ev) CK(cudaEventCreate(&e));
+        struct EvGuard { cudaEvent_t *e; ~EvGuard() { for (int i = 0; i < 5; ++i) if (e[i]) cudaEventDestroy(e[i]); } } evg{ev};
         CK(cudaMalloc(&c->d_kc, sizeof(double) * kc.size()));
         CK(cudaMemcpy(c->d_kc, kc.data(), sizeof(double) * kc.size(), cudaMemcpyHostToDevice));
         CK(cudaMalloc(&c->d_cnt, 8 * sizeof(unsigned long long)));
         CK(cudaMalloc(&c->d_tile_counter, sizeof(int)));
         c->num_sms = prop.multiProcessorCount;
-        CK(cudaMemset(c->d_cnt, 0, 8 * sizeof(unsigned long long)));
+        CK(cudaMemsetAsync(c->d_cnt, 0, 8 * sizeof(unsigned long long), c->stream));
         const int64_t ncell = (int64_t)c->ncx * c->ncy;
         CK(cudaMalloc(&c->d_cell_start, sizeof(int) * (ncell + 1)));
         if (nt == 0) {
-            CK(cudaMemset(c->d_cell_start, 0, sizeof(int) * (ncell + 1)));
+            CK(cudaMemsetAsync(c->d_cell_start, 0, sizeof(int) * (ncell + 1), c->stream));
+            CK(cudaStreamSynchronize(c->stream));
+            c->cinfo.device_bytes = (int64_t)(sizeof(int) * (ncell + 1) + sizeof(double) * kc.size() + 64 + 4);
+            c->cinfo.total_ms = ms_since(t_start);
             return;
         }
         const int rs = (16 + nb + 1) & ~1;
@@ -482,24 +514,27 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
             }
             CK(cudaMalloc(&c->d_rec, sizeof(double) * rs * nt));
             CK(cudaMalloc(&c->d_bbox, sizeof(double4) * nt));
-            CK(cudaMemcpy(dV, V, sizeof(double) * 2 * nv, cudaMemcpyHostToDevice));
-            CK(cudaMemcpy(dT, T, sizeof(int) * 3 * nt, cudaMemcpyHostToDevice));
-            CK(cudaMemcpy(dC, C, sizeof(double) * nb * nt, cudaMemcpyHostToDevice));
-            CK(cudaMemcpy(dR, R.data(), sizeof(double) * nb * nb, cudaMemcpyHostToDevice));
-            PrepArgs pa{dV, dT, dC, dR, nt, nb, rs, p->h, p->domain[0], p->domain[1], c->cw, c->chh,
-                        c->ncx, c->ncy, rec_u, bb_u, keys[0], idx[0]};
-            k_prep<<<nblk(nt, 256), 256>>>(pa);
-            CK(cudaGetLastError());
             cub::DoubleBuffer<uint32_t> kb(keys[0], keys[1]);
             cub::DoubleBuffer<int> vb(idx[0], idx[1]);
             size_t bytes = 0;
             CK(cub::DeviceRadixSort::SortPairs(nullptr, bytes, kb, vb, (int)nt));
             CK(cudaMalloc(&tmp, bytes));
-            CK(cub::DeviceRadixSort::SortPairs(tmp, bytes, kb, vb, (int)nt));
-            k_gather<<<nblk(nt, 256), 256>>>(rec_u, bb_u, vb.Current(), nt, rs, c->d_rec, c->d_bbox);
+            CK(cudaEventRecord(ev[0], cs));
+            CK(cudaMemcpyAsync(dV, V, sizeof(double) * 2 * nv, cudaMemcpyHostToDevice, cs));
+            CK(cudaMemcpyAsync(dT, T, sizeof(int) * 3 * nt, cudaMemcpyHostToDevice, cs));
+            CK(cudaMemcpyAsync(dC, C, sizeof(double) * nb * nt, cudaMemcpyHostToDevice, cs));
+            CK(cudaMemcpyAsync(dR, R.data(), sizeof(double) * nb * nb, cudaMemcpyHostToDevice, cs));
+            CK(cudaEventRecord(ev[1], cs));
+            PrepArgs pa{dV, dT, dC, dR, nt, nb, rs, p->h, p->domain[0], p->domain[1], c->cw, c->chh,
+                        c->ncx, c->ncy, rec_u, bb_u, keys[0], idx[0]};
+            k_prep<<<nblk(nt, 256), 256, 0, cs>>>(pa);
             CK(cudaGetLastError());
-            k_cell_start<<<nblk(ncell + 1, 256), 256>>>(kb.Current(), nt, ncell, c->d_cell_start);
+            CK(cub::DeviceRadixSort::SortPairs(tmp, bytes, kb, vb, (int)nt, 0, sizeof(uint32_t) * 8, cs));
+            k_gather<<<nblk(nt, 256), 256, 0, cs>>>(rec_u, bb_u, vb.Current(), nt, rs, c->d_rec, c->d_bbox);
             CK(cudaGetLastError());
+            k_cell_start<<<nblk(ncell + 1, 256), 256, 0, cs>>>(kb.Current(), nt, ncell, c->d_cell_start);
+            CK(cudaGetLastError());
+            CK(cudaEventRecord(ev[2], cs));
             // schedule JUMP: per-triangle moments and corner polynomials (siac_jump.cuh)
             int jrs = 0;
             switch (k) {
@@ -510,11 +545,12 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
             }
             CK(cudaMalloc(&c->d_jrec, sizeof(double) * jrs * nt));
             switch (k) {
-                case 1: CK(siac_prep_jump_k1(c->d_rec, nt, p->h, c->d_jrec)); break;
-                case 2: CK(siac_prep_jump_k2(c->d_rec, nt, p->h, c->d_jrec)); break;
-                case 3: CK(siac_prep_jump_k3(c->d_rec, nt, p->h, c->d_jrec)); break;
-                default: CK(siac_prep_jump_k4(c->d_rec, nt, p->h, c->d_jrec)); break;
+                case 1: CK(siac_prep_jump_k1(c->d_rec, nt, p->h, c->d_jrec, cs)); break;
+                case 2: CK(siac_prep_jump_k2(c->d_rec, nt, p->h, c->d_jrec, cs)); break;
+                case 3: CK(siac_prep_jump_k3(c->d_rec, nt, p->h, c->d_jrec, cs)); break;
+                default: CK(siac_prep_jump_k4(c->d_rec, nt, p->h, c->d_jrec, cs)); break;
             }
+            CK(cudaEventRecord(ev[3], cs));
             // closed-form cross terms (interval polynomials of the reference corners)
             int xrs = 0;
             switch (k) {
@@ -525,18 +561,33 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
             }
             CK(cudaMalloc(&c->d_xrec, sizeof(double) * xrs * nt));
             switch (k) {
-                case 1: CK(siac_prep_cross_k1(c->d_jrec, nt, c->d_xrec)); break;
-                case 2: CK(siac_prep_cross_k2(c->d_jrec, nt, c->d_xrec)); break;
-                case 3: CK(siac_prep_cross_k3(c->d_jrec, nt, c->d_xrec)); break;
-                default: CK(siac_prep_cross_k4(c->d_jrec, nt, c->d_xrec)); break;
+                case 1: CK(siac_prep_cross_k1(c->d_jrec, nt, c->d_xrec, cs)); break;
+                case 2: CK(siac_prep_cross_k2(c->d_jrec, nt, c->d_xrec, cs)); break;
+                case 3: CK(siac_prep_cross_k3(c->d_jrec, nt, c->d_xrec, cs)); break;
+                default: CK(siac_prep_cross_k4(c->d_jrec, nt, c->d_xrec, cs)); break;
             }
             CK(cudaGetLastError());
-            CK(cudaDeviceSynchronize());
+            CK(cudaEventRecord(ev[4], cs));
+            CK(cudaStreamSynchronize(cs));
+            float t01 = 0, t12 = 0, t23 = 0, t34 = 0;
+            CK(cudaEventElapsedTime(&t01, ev[0], ev[1]));
+            CK(cudaEventElapsedTime(&t12, ev[1], ev[2]));
+            CK(cudaEventElapsedTime(&t23, ev[2], ev[3]));
+            CK(cudaEventElapsedTime(&t34, ev[3], ev[4]));
+            c->cinfo.h2d_ms = t01;
+            c->cinfo.index_ms = t12;
+            c->cinfo.jump_ms = t23;
+            c->cinfo.cross_ms = t34;
+            const int64_t per_tri = (int64_t)sizeof(double) * (rs + jrs + xrs) + (int64_t)sizeof(double4);
+            c->cinfo.bytes_per_triangle = per_tri;
+            c->cinfo.device_bytes = per_tri * nt + (int64_t)sizeof(int) * (ncell + 1) +
+                                    (int64_t)(sizeof(double) * kc.size()) + 64 + 4;
         } catch (...) {
             cleanup();
             throw;
         }
         cleanup();
+        c->cinfo.total_ms = ms_since(t_start);
     });
     if (st != SIAC_OK) {
         free_ctx(c);
@@ -568,7 +619,11 @@ siac_status siac_eval_async(siac_ctx *ctx, const double *d_pts, int64_t np, doub
                 CK(cudaGraphLaunch(g.exec, st));
                 return;
             }
-        if (ctx->gcache.empty()) eval_device(ctx, d_pts, np, d_out, st);   // first use: kernel attributes
+        // The very first evaluation of a context runs directly (it sets the kernels' shared-memory
+        // attributes and loads the modules, which must not happen inside a capture) and is this
+        // call's result; the graph captured right after is only instantiated, not launched.
+        const bool first = ctx->gcache.empty();
+        if (first) eval_device(ctx, d_pts, np, d_out, st);
         cudaGraph_t graph = nullptr;
         CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed));
         try {
@@ -588,7 +643,7 @@ siac_status siac_eval_async(siac_ctx *ctx, const double *d_pts, int64_t np, doub
             ctx->gcache.erase(ctx->gcache.begin());
         }
         ctx->gcache.push_back({d_pts, np, d_out, ctx->schedule, exec});
-        CK(cudaGraphLaunch(exec, st));
+        if (!first) CK(cudaGraphLaunch(exec, st));
     });
 }
 
@@ -618,7 +673,7 @@ siac_status siac_eval(siac_ctx *ctx, const double *pts, int64_t np, double *out)
             CK(cudaMalloc(&ctx->d_hout, sizeof(double) * np));
             ctx->cap_host = np;
         }
-        cudaStream_t st = 0;
+        cudaStream_t st = ctx->stream;
         CK(cudaMemcpyAsync(ctx->d_hpts, pts, sizeof(double) * 2 * np, cudaMemcpyHostToDevice, st));
         eval_device(ctx, ctx->d_hpts, np, ctx->d_hout, st);
         CK(cudaMemcpyAsync(out, ctx->d_hout, sizeof(double) * np, cudaMemcpyDeviceToHost, st));
@@ -632,8 +687,15 @@ siac_status siac_set_counting(siac_ctx *ctx, int32_t enable) {
     return SIAC_OK;
 }
 
-siac_status siac_stats(siac_ctx *ctx, siac_counters *out) {
+siac_status siac_get_create_info(const siac_ctx *ctx, siac_create_info *out) {
     if (!ctx || !out) { g_err = "NULL argument"; return SIAC_EINVAL; }
+    *out = ctx->cinfo;
+    return SIAC_OK;
+}
+
+siac_status siac_stats(const siac_ctx *cctx, siac_counters *out) {
+    if (!cctx || !out) { g_err = "NULL argument"; return SIAC_EINVAL; }
+    siac_ctx *ctx = const_cast<siac_ctx *>(cctx);     // only the error message is written
     return run_guarded(&ctx->err, [&]() {
         CK(cudaSetDevice(ctx->device));
         unsigned long long h[8];

@@ -220,12 +220,12 @@ cudaError_t SIAC_FN(SIAC_K, SIAC_PART)(const EvalArgs &a, bool count, int *tile_
 }
 
 #if SIAC_PART == 0
-cudaError_t SIAC_CAT(siac_prep_jump_k, SIAC_K)(const double *rec, int64_t nt, double h, double *jrec) {
-    siacjump::k_prep_jump<SIAC_K><<<(unsigned)((nt + 127) / 128), 128>>>(rec, nt, h, jrec);
+cudaError_t SIAC_CAT(siac_prep_jump_k, SIAC_K)(const double *rec, int64_t nt, double h, double *jrec, cudaStream_t st) {
+    siacjump::k_prep_jump<SIAC_K><<<(unsigned)((nt + 127) / 128), 128, 0, st>>>(rec, nt, h, jrec);
     return cudaGetLastError();
 }
-cudaError_t SIAC_CAT(siac_prep_cross_k, SIAC_K)(const double *jrec, int64_t nt, double *xrec) {
-    siacjump::k_prep_cross<SIAC_K><<<(unsigned)((4 * nt + 127) / 128), 128>>>(jrec, nt, xrec);
+cudaError_t SIAC_CAT(siac_prep_cross_k, SIAC_K)(const double *jrec, int64_t nt, double *xrec, cudaStream_t st) {
+    siacjump::k_prep_cross<SIAC_K><<<(unsigned)((4 * nt + 127) / 128), 128, 0, st>>>(jrec, nt, xrec);
     return cudaGetLastError();
 }
 int SIAC_CAT(siac_xrec_doubles_k, SIAC_K)() { return siacjump::XRec<SIAC_K>::RS; }

@@ -35,8 +35,8 @@ struct EvalArgs {            // arguments of every evaluation schedule
                                              int num_sms, cudaStream_t st);
 #define SIAC_DECL_K(k)                                                                          \
     SIAC_DECL_KP(k, 0) SIAC_DECL_KP(k, 1) SIAC_DECL_KP(k, 2) SIAC_DECL_KP(k, 3)                 \
-    cudaError_t siac_prep_jump_k##k(const double *rec, int64_t nt, double h, double *jrec);        \
-    cudaError_t siac_prep_cross_k##k(const double *jrec, int64_t nt, double *xrec);                \
+    cudaError_t siac_prep_jump_k##k(const double *rec, int64_t nt, double h, double *jrec, cudaStream_t st); \
+    cudaError_t siac_prep_cross_k##k(const double *jrec, int64_t nt, double *xrec, cudaStream_t st);         \
     cudaError_t siac_launch_elem_k##k(const EvalArgs &a, bool count, int *, int, cudaStream_t st); \
     int siac_xrec_doubles_k##k();
 SIAC_DECL_K(1)

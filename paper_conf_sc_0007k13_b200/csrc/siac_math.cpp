@@ -264,4 +264,21 @@ std::vector<double> dubiner_to_centred(int k, std::vector<std::pair<int, int>> *
     return R;
 }
 
+std::vector<double> monomial_to_centred(int k) {
+    std::vector<std::pair<int, int>> order;
+    dubiner_to_centred(k, &order);
+    const int nb = (k + 1) * (k + 2) / 2;
+    std::vector<double> R((size_t)nb * nb, 0.0);
+    const Q third = Q::frac(1, 3);
+    const P2 rr = p2_lin(k, third, third, Q(0));      // r = (rho + 1)/3
+    const P2 ss = p2_lin(k, third, Q(0), third);      // s = (sigma + 1)/3
+    int i = 0;
+    for (int n = 0; n <= k; ++n)
+        for (int b = 0; b <= n; ++b, ++i) {
+            const P2 m = p2_mul(p2_pow(rr, n - b), p2_pow(ss, b));
+            for (int j = 0; j < nb; ++j) R[(size_t)i * nb + j] = m.at(order[j].first, order[j].second).to_double();
+        }
+    return R;
+}
+
 }  // namespace siac

@@ -13,4 +13,8 @@ std::vector<double> kernel_cell_table(int k, std::vector<double> *coeffs_out = n
 // Row-major nb x nb: row i = orthonormal Dubiner mode i in centred monomials, device Horner order.
 std::vector<double> dubiner_to_centred(int k, std::vector<std::pair<int, int>> *order_out = nullptr);
 
+// Same layout for SIAC_BASIS_MONOMIAL_REF: row i = r^a s^b (i by n = a + b, then b) in the
+// centred monomials (r = (rho + 1)/3, s = (sigma + 1)/3), exact rationals rounded once.
+std::vector<double> monomial_to_centred(int k);
+
 }  // namespace siac

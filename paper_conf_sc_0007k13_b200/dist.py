@@ -131,6 +131,44 @@ def halo(V, T, points, half_width, domain=(0.0, 0.0, 1.0, 1.0), periodic: int = 
     return np.nonzero(keep)[0]
 
 
+def near_cut_points(points, part: dict, half_width: float) -> np.ndarray:
+    """Indices (ascending) of the points whose stencil square (half-width `half_width`) reaches
+    a cell holding points of another rank: the points whose values depend on the halo
+    (parity "plus points within W of partition boundaries").  Cell test on a
+    grid of cells >= half_width, wrapping on periodic axes; conservative."""
+    x0, y0, x1, y1 = part["domain"]
+    periodic = part["periodic"]
+    P = wrap_points(points, part["domain"], periodic)
+    nx = max(1, int((x1 - x0) / half_width))
+    ny = max(1, int((y1 - y0) / half_width))
+    ix = np.clip(((P[:, 0] - x0) / (x1 - x0) * nx).astype(np.int64), 0, nx - 1)
+    iy = np.clip(((P[:, 1] - y0) / (y1 - y0) * ny).astype(np.int64), 0, ny - 1)
+    owner = np.empty(len(P), dtype=np.int64)
+    for r in range(part["world"]):
+        owner[part["order"][part["bounds"][r]:part["bounds"][r + 1]]] = r
+    lo = np.full((ny, nx), part["world"], dtype=np.int64)
+    hi = np.full((ny, nx), -1, dtype=np.int64)
+    np.minimum.at(lo, (iy, ix), owner)
+    np.maximum.at(hi, (iy, ix), owner)
+    near = np.zeros(len(P), dtype=bool)
+    for dj in (-1, 0, 1):
+        for di in (-1, 0, 1):
+            jj, ii = iy + dj, ix + di
+            ok = np.ones(len(P), dtype=bool)
+            if periodic & 1:
+                ii = ii % nx
+            else:
+                ok &= (ii >= 0) & (ii < nx)
+            if periodic & 2:
+                jj = jj % ny
+            else:
+                ok &= (jj >= 0) & (jj < ny)
+            jj, ii = np.clip(jj, 0, ny - 1), np.clip(ii, 0, nx - 1)
+            other = ok & (((lo[jj, ii] != owner) & (lo[jj, ii] < part["world"])) | ((hi[jj, ii] != owner) & (hi[jj, ii] >= 0)))
+            near |= other
+    return np.nonzero(near)[0]
+
+
 def local_problem(V, T, C, points, k: int, h: float, part: dict, rank: int) -> dict:
     """The rank's points (in partition order) and its halo triangles."""
     lo, hi = part["bounds"][rank], part["bounds"][rank + 1]

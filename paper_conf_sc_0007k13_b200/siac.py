@@ -32,6 +32,10 @@ NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a",
 
 SIAC_PERIODIC_X = 1
 SIAC_PERIODIC_Y = 2
+SIAC_BASIS_DUBINER_ORTHONORMAL = 0
+SIAC_BASIS_MONOMIAL_REF = 1
+SIAC_BOUNDARY_ZERO = 0
+SIAC_BOUNDARY_ONESIDED = 1
 
 
 def build(force: bool = False, verbose: bool = False, extra_flags=(), out_path: str | None = None) -> str:
@@ -102,7 +106,14 @@ class SiacError(RuntimeError):
 
 class _Params(ctypes.Structure):
     _fields_ = [("k", ctypes.c_int32), ("h", ctypes.c_double), ("periodic", ctypes.c_int32),
-                ("domain", ctypes.c_double * 4), ("device", ctypes.c_int32), ("cell_factor", ctypes.c_double)]
+                ("domain", ctypes.c_double * 4), ("device", ctypes.c_int32), ("cell_factor", ctypes.c_double),
+                ("basis", ctypes.c_int32), ("boundary", ctypes.c_int32)]
+
+
+class _CreateInfo(ctypes.Structure):
+    _fields_ = [("total_ms", ctypes.c_double), ("host_ms", ctypes.c_double), ("h2d_ms", ctypes.c_double),
+                ("index_ms", ctypes.c_double), ("jump_ms", ctypes.c_double), ("cross_ms", ctypes.c_double),
+                ("device_bytes", ctypes.c_int64), ("bytes_per_triangle", ctypes.c_int64)]
 
 
 class _Counters(ctypes.Structure):
@@ -133,6 +144,8 @@ def lib():
         L.siac_set_counting.argtypes = [vp, I32]
         L.siac_stats.restype = ctypes.c_int
         L.siac_stats.argtypes = [vp, ctypes.POINTER(_Counters)]
+        L.siac_get_create_info.restype = ctypes.c_int
+        L.siac_get_create_info.argtypes = [vp, ctypes.POINTER(_CreateInfo)]
         L.siac_set_schedule.restype = ctypes.c_int
         L.siac_set_schedule.argtypes = [vp, I32]
         L.siac_set_graphs.restype = ctypes.c_int
@@ -168,7 +181,7 @@ def lib():
     return _lib
 
 
-EXPORTED = ["siac_create", "siac_eval", "siac_eval_async", "siac_set_counting", "siac_stats",
+EXPORTED = ["siac_create", "siac_eval", "siac_eval_async", "siac_set_counting", "siac_stats", "siac_get_create_info",
             "siac_set_schedule", "siac_set_graphs", "siac_set_timing", "siac_timing", "siac_probe_fp64",
             "siac_info", "siac_host_tables", "siac_debug_records",
             "siac_destroy", "siac_last_error", "siac_version",
@@ -189,12 +202,15 @@ class Context:
     """A siac_ctx: device-resident mesh + spatial index."""
 
     def __init__(self, V, T, C, k: int, h: float, periodic: int = 3, domain=(0.0, 0.0, 1.0, 1.0),
-                 device: int = 0, cell_factor: float = 0.0):
+                 device: int = 0, cell_factor: float = 0.0, basis: int = 0, boundary: int = 0):
         L = lib()
-        self._V = np.ascontiguousarray(V, dtype=np.float64)
-        self._T = np.ascontiguousarray(T, dtype=np.int32)
+        self._V = np.ascontiguousarray(V, dtype=np.float64).reshape(-1, 2)
+        self._T = np.ascontiguousarray(T, dtype=np.int32).reshape(-1, 3)
         self._C = np.ascontiguousarray(C, dtype=np.float64)
-        p = _Params(int(k), float(h), int(periodic), (ctypes.c_double * 4)(*domain), int(device), float(cell_factor))
+        if 1 <= k <= 4 and self._C.size != len(self._T) * (k + 1) * (k + 2) // 2:   # (k itself: checked in C)
+            raise ValueError(f"coeffs must have (k+1)(k+2)/2 = {(k + 1) * (k + 2) // 2} columns")
+        p = _Params(int(k), float(h), int(periodic), (ctypes.c_double * 4)(*domain), int(device), float(cell_factor),
+                    int(basis), int(boundary))
         ptr = ctypes.c_void_p()
         rc = L.siac_create(ctypes.byref(ptr), _dp(self._V), len(self._V),
                            self._T.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)), len(self._T),
@@ -212,7 +228,14 @@ class Context:
         return out
 
     def eval_into(self, points: np.ndarray, out: np.ndarray) -> None:
-        """siac_eval into caller-owned host arrays (e.g. pinned torch tensors' numpy views)."""
+        """siac_eval into caller-owned host arrays (e.g. pinned torch tensors' numpy views).
+        points: float64, C-contiguous, shape (n, 2); out: float64, C-contiguous, >= n values."""
+        if not (isinstance(points, np.ndarray) and points.dtype == np.float64 and points.flags.c_contiguous
+                and points.ndim == 2 and points.shape[1] == 2):
+            raise ValueError("points must be a C-contiguous float64 array of shape (n, 2)")
+        if not (isinstance(out, np.ndarray) and out.dtype == np.float64 and out.flags.c_contiguous
+                and out.size >= len(points)):
+            raise ValueError("out must be a C-contiguous float64 array with at least n values")
         _check(lib().siac_eval(self._ptr, _dp(points), len(points), _dp(out)), self._ptr)
 
     def eval_async(self, d_points, d_out, stream=None) -> None:
@@ -246,6 +269,12 @@ class Context:
         c = _Counters()
         _check(lib().siac_stats(self._ptr, ctypes.byref(c)), self._ptr)
         return {f: getattr(c, f) for f, _ in _Counters._fields_}
+
+    def create_info(self) -> dict:
+        """siac_get_create_info: siac_create's cost (ms per stage) and resident device bytes."""
+        c = _CreateInfo()
+        _check(lib().siac_get_create_info(self._ptr, ctypes.byref(c)), self._ptr)
+        return {f: getattr(c, f) for f, _ in _CreateInfo._fields_}
 
     def set_schedule(self, schedule: int) -> None:
         """0 = default (fastest = 5), 1 = thread-per-point, 2 = warp-per-tile, 3 = warp-specialized, 4 = jump,
@@ -297,8 +326,9 @@ class Context:
         self.destroy()
 
 
-def create(V, T, C, k, h, periodic=3, domain=(0.0, 0.0, 1.0, 1.0), device=0, cell_factor=0.0) -> Context:
-    return Context(V, T, C, k, h, periodic, domain, device, cell_factor)
+def create(V, T, C, k, h, periodic=3, domain=(0.0, 0.0, 1.0, 1.0), device=0, cell_factor=0.0, basis=0,
+           boundary=0) -> Context:
+    return Context(V, T, C, k, h, periodic, domain, device, cell_factor, basis, boundary)
 
 
 def host_tables(k: int):

@@ -49,7 +49,7 @@ def _params(**kw):
 @pytest.mark.parametrize("bad,msg", [
     (dict(k=0), "k must"), (dict(k=5), "k must"), (dict(h=-1.0), "h must"), (dict(h=float("nan")), "h must"),
     (dict(h=0.3), "exceeds the periodic"), (dict(domain=(0.0, 0.0, -1.0, 1.0)), "domain"),
-    (dict(periodic=4), "periodic"),
+    (dict(periodic=4), "periodic"), (dict(basis=2), "basis"), (dict(boundary=2), "boundary"),
 ])
 def test_create_rejects_bad_params(L, bad, msg):
     V, T = inputs.structured_mesh(4)

@@ -145,3 +145,51 @@ def test_work_estimate_tracks_pair_counts_and_balances_graded_mesh():
         tot = [est[part["order"][part["bounds"][r]:part["bounds"][r + 1]]].sum() for r in range(world)]
         spread[name] = max(tot) / min(tot)
     assert spread["work"] < 1.01 and spread["count"] > 1.5
+
+
+def _bcast_worker(rank, world, port, out_path):
+    import torch
+    import torch.distributed as dist
+
+    import bench
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    w = inputs.make_config(2) if rank == 0 else None
+    got, ms = bench.broadcast_workload(w, rank, torch.device("cpu"))
+    if rank == 1:
+        np.savez(out_path, V=got.V, T=got.T, C=got.C, P=got.points, k=got.k, h=got.h, n=got.n_points)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_bench_broadcasts_rank0_workload(tmp_path):
+    """bench.py N > 1: rank 0 generates the workload once and broadcasts it (SURVEY §3.5);
+    rank 1 receives bitwise the same mesh, modes and points (gloo, world 2)."""
+    import torch.multiprocessing as mp
+    out = str(tmp_path / "w.npz")
+    mp.spawn(_bcast_worker, args=(2, _free_port(), out), nprocs=2, join=True)
+    got = np.load(out)
+    w = inputs.make_config(2)
+    for a, b in ((got["V"], w.V), (got["T"], w.T), (got["C"], w.C), (got["P"], w.points)):
+        assert a.dtype == b.dtype and np.array_equal(a, b)
+    assert int(got["k"]) == w.k and float(got["h"]) == w.h and int(got["n"]) == w.n_points
+
+
+def test_near_cut_points_cover_halo_dependent_points():
+    """dist.near_cut_points contains every point with a point of another rank inside its
+    stencil square (brute force on a sample), and is a proper subset on a fine mesh."""
+    w = inputs.make_config(3)
+    hw = 0.5 * (3 * w.k + 1) * w.h
+    part = sdist.partition(w.points, 8)
+    near = set(sdist.near_cut_points(w.points, part, hw).tolist())
+    owner = np.empty(w.n_points, dtype=np.int64)
+    for r in range(8):
+        owner[part["order"][part["bounds"][r]:part["bounds"][r + 1]]] = r
+    rng = np.random.default_rng(3)
+    for i in rng.choice(w.n_points, 400, replace=False):
+        d = np.abs(w.points - w.points[i])
+        d = np.minimum(d, 1 - d)
+        if np.any((d.max(axis=1) < hw) & (owner != owner[i])):
+            assert i in near
+    assert len(sdist.near_cut_points(w.points, part, 0.02)) < 0.5 * w.n_points   # narrow stencil: a subset

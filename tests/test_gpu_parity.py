@@ -358,3 +358,79 @@ def test_graph_replay_matches_direct(siac_mod, sch):
                     assert np.array_equal(g, r)
     ctx.set_graphs(False)
     ctx.destroy()
+
+
+# ------------------------------------------------------------------ full-size cross-checks (round 2)
+
+def test_cfg5_jumpx_equals_tile_every_point(siac_mod):
+    """Config 5 (1.05M triangles, P3, 12.6M points): the default schedule (JUMPX, spline-jump
+    decomposition in closed form) against the direct clip-and-integrate schedule (TILE:
+    Sutherland-Hodgman pieces, fan, degree-3k quadrature, Eq. (2) literally) at EVERY point,
+    both in the bench's launch configuration.  Two unrelated decompositions of the same
+    integral; the oracle pins the sample (test_large_configs_sampled)."""
+    for field in ("sinsin", "random"):
+        w = cfg(5, field)
+        ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
+        gj = ctx.eval(w.points)
+        ctx.set_schedule(2)
+        gt = ctx.eval(w.points)
+        ctx.destroy()
+        assert_parity(gj, gt)
+        err = np.abs(gj - gt).max() / np.abs(gt).max()
+        print(f"cfg5 {field}: JUMPX vs TILE normwise {err:.2e} over {w.n_points} points")
+        assert err <= 1e-12
+
+
+@pytest.mark.parametrize("c", [3, 5])
+def test_partitioned_equals_single_gpu(siac_mod, c):
+    """The multi-GPU split: for G = 2, 4, 8 ranks,
+    dist.partition (Morton ranges of equal estimated work) + dist.local_problem (triangle halo)
+    + one siac_create per partition, evaluated one after the other on this GPU and assembled,
+    equals the single-context result at every point (only the summation grouping differs)."""
+    from paper_conf_sc_0007k13_b200 import dist as sdist
+    w = cfg(c, "random")
+    ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
+    ref = ctx.eval(w.points)
+    ctx.destroy()
+    hw = 0.5 * (3 * w.k + 1) * w.h
+    wts = sdist.work_estimate(w.V, w.T, w.points, hw)
+    for G in (2, 4, 8):
+        part = sdist.partition(w.points, G, weights=wts)
+        gathered = np.zeros((G, part["max_count"]))
+        for r in range(G):
+            loc = sdist.local_problem(w.V, w.T, w.C, w.points, w.k, w.h, part, r)
+            assert len(loc["triangles"]) < len(w.T) or G == 2
+            cr = siac_mod.create(loc["V"], loc["T"], loc["C"], w.k, w.h)
+            gathered[r, :len(loc["points"])] = cr.eval(loc["points"])
+            cr.destroy()
+        got = sdist.assemble(gathered.ravel(), part, w.n_points)
+        err = np.abs(got - ref).max() / np.abs(ref).max()
+        print(f"cfg{c} G={G}: normwise {err:.2e}")
+        assert err <= 1e-13
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 4])
+def test_monomial_ref_basis(siac_mod, oracle_mod, k):
+    """params.basis = SIAC_BASIS_MONOMIAL_REF against the oracle's plain
+    per-triangle monomial field (field_mode 2)."""
+    V, T = inputs.lattice_delaunay_mesh(1500, seed=40 + k)
+    M = np.random.default_rng(k).uniform(-1, 1, (len(T), inputs.n_modes(k)))
+    h = inputs.max_edge(V, T)
+    P = inputs.eval_points(V, T, k)[::7]
+    ctx = siac_mod.create(V, T, M, k, h, basis=siac_mod.SIAC_BASIS_MONOMIAL_REF)
+    g = ctx.eval(P)
+    ctx.destroy()
+    assert_parity(g, oracle_mod.oracle_eval(V, T, M, k, h, P, field_mode=2))
+
+
+def test_create_info(siac_mod):
+    """siac_get_create_info: stage times and the resident footprint of siac_create."""
+    w = cfg(2)
+    ctx = siac_mod.create(w.V, w.T, w.C, w.k, w.h)
+    ci = ctx.create_info()
+    ctx.destroy()
+    for f in ("host_ms", "h2d_ms", "index_ms", "jump_ms", "cross_ms"):
+        assert ci[f] >= 0.0
+    assert ci["total_ms"] >= ci["h2d_ms"] + ci["index_ms"] + ci["jump_ms"] + ci["cross_ms"]
+    assert ci["bytes_per_triangle"] > 8 * inputs.n_modes(w.k)
+    assert ci["device_bytes"] >= ci["bytes_per_triangle"] * len(w.T)

@@ -53,3 +53,62 @@ def test_dubiner_at_top_vertex_finite(oracle_mod, k):
     """The collapsed recurrence has no division by (1 - eta): finite at eta = 1."""
     v = oracle_mod.dubiner_values(k, np.array([-1.0]), np.array([1.0]))
     assert np.all(np.isfinite(v))
+
+
+# ------------------------------------------------------------------ SIAC_BASIS_MONOMIAL_REF
+# (SURVEY §8(b): params.basis, "Sum c_ab r^a s^b on the unit reference triangle, offered for
+# tests"; the oracle's field_mode 2)
+
+def _mons(k):
+    return [(n - b, b) for n in range(k + 1) for b in range(n + 1)]
+
+
+def monomial_ref_coeffs(V, T, k, f):
+    """Per-triangle coefficients of r^a s^b interpolating f at the lattice points (i/k, j/k)
+    of the unit reference triangle (unisolvent for P_k): exact for f in P_k.  Input
+    generation only (a Vandermonde solve), no SIAC arithmetic."""
+    mons = _mons(k)
+    rs = np.array([(i / k, j / k) for j in range(k + 1) for i in range(k + 1 - j)])
+    A = np.stack([rs[:, 0] ** a * rs[:, 1] ** b for a, b in mons], axis=1)
+    v0, v1, v2 = V[T[:, 0]], V[T[:, 1]], V[T[:, 2]]
+    X = v0[:, None, :] + rs[None, :, 0, None] * (v1 - v0)[:, None, :] + rs[None, :, 1, None] * (v2 - v0)[:, None, :]
+    F = f(X[..., 0], X[..., 1])
+    return np.linalg.solve(A[None], F[..., None])[..., 0]
+
+
+def monomial_to_dubiner(M, k, n_quad=None):
+    """L2 projection onto the orthonormal Dubiner modes of sum_i M[t, i] r^a s^b (the input
+    generator's collapsed rule and scipy Dubiner values; exact for degree k)."""
+    xi, eta, W = inputs._ref_rule(n_quad or k + 2)
+    Phi = inputs.dubiner_eval(k, xi, eta)
+    r, s = (xi + 1) / 2, (eta + 1) / 2
+    B = np.stack([r ** a * s ** b for a, b in _mons(k)], axis=1)       # (nq, nb)
+    return ((M @ B.T) * W[None, :]) @ Phi
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 4])
+def test_monomial_basis_reproduces_global_polynomial(oracle_mod, k):
+    """u_h = a global polynomial of degree k written in per-triangle reference monomials ->
+    u* = u at interior points (degree <= 2k reproduction, L202-205)."""
+    V, T = inputs.lattice_delaunay_mesh(700, seed=8)
+    f = lambda x, y: 0.3 - (x + 0.2 * y) ** k + 0.5 * x ** (k - 1) * y  # noqa: E731
+    M = monomial_ref_coeffs(V, T, k, f)
+    h = 0.03
+    W = (3 * k + 1) * h
+    P = np.random.default_rng(3).uniform(W / 2 + 0.01, 1 - W / 2 - 0.01, (10, 2))
+    u = oracle_mod.oracle_eval(V, T, M, k, h, P, periodic=0, field_mode=2)
+    assert np.abs(u - f(P[:, 0], P[:, 1])).max() < 1e-12
+
+
+@pytest.mark.parametrize("k", [1, 3])
+def test_monomial_basis_equals_dubiner_random_field(oracle_mod, k):
+    """A random per-triangle field in reference monomials == the same field projected onto
+    the Dubiner basis (two independent field evaluations inside the oracle)."""
+    w = inputs.make_config(2)
+    V, T = w.V, w.T
+    M = np.random.default_rng(4).uniform(-1, 1, (len(T), inputs.n_modes(k)))
+    D = monomial_to_dubiner(M, k)
+    P = w.points[::211]
+    u2 = oracle_mod.oracle_eval(V, T, M, k, w.h, P, field_mode=2)
+    u0 = oracle_mod.oracle_eval(V, T, D, k, w.h, P)
+    assert np.abs(u2 - u0).max() < 1e-12 * np.abs(u0).max()
