@@ -49,8 +49,9 @@ def _load():
         D, L, I = ctypes.POINTER(ctypes.c_double), ctypes.c_long, ctypes.c_int
         lib.oracle_siac_eval.restype = I
         lib.oracle_siac_eval.argtypes = [I, ctypes.c_double, I, D, D, L, ctypes.POINTER(ctypes.c_int), L,
-                                         I, D, I, D, I, D, D, I, D, D, D, L, D, D, I, I]
+                                         I, D, I, D, I, D, D, I, D, D, D, L, D, D, I, I, D, D]
         lib.oracle_kernel_many.argtypes = [I, D, D, L, D]
+        lib.oracle_kernel_shifted_many.argtypes = [I, D, ctypes.c_double, D, L, D]
         lib.oracle_bspline_many.argtypes = [I, D, L, D]
         lib.oracle_dubiner_many.argtypes = [I, D, D, L, D]
         _lib = lib
@@ -111,6 +112,51 @@ def kernel_coefficients(k: int) -> list[Fraction]:
     return [M[i][n] for i in range(n)]
 
 
+def kernel_coefficients_shifted(k: int, lam) -> list[Fraction]:
+    """The one-sided kernel of ref [21] (Ryan & Shu 2003; "an asymmetric
+    (one-sided) stencil is used [21]"; reading R4): the 2k+1 B-spline nodes shifted to
+    x_g = -k + g + lambda, the coefficients solving the SAME moment conditions as the symmetric
+    kernel at the shifted nodes,
+        int K(t) dt = 1,   int K(t) t^m dt = 0,  m = 1..2k,
+    by exact Gauss-Jordan over the rationals (lambda converted exactly from its double)."""
+    lam = Fraction(lam)
+    n = 2 * k + 1
+    mu = [bspline_moments(k, l) for l in range(n)]
+    xg = [Fraction(g - k) + lam for g in range(n)]
+    A = [[sum(math.comb(m, l) * xg[g] ** (m - l) * mu[l] for l in range(m + 1)) for g in range(n)]
+         for m in range(n)]
+    M = [row[:] + [Fraction(1 if i == 0 else 0)] for i, row in enumerate(A)]
+    for col in range(n):
+        piv = next(r for r in range(col, n) if M[r][col] != 0)
+        M[col], M[piv] = M[piv], M[col]
+        pv = M[col][col]
+        M[col] = [v / pv for v in M[col]]
+        for r in range(n):
+            if r != col and M[r][col] != 0:
+                f = M[r][col]
+                M[r] = [a - f * c for a, c in zip(M[r], M[col])]
+    return [M[i][n] for i in range(n)]
+
+
+def onesided_shift(k: int, h: float, x, lo: float, hi: float):
+    """Node shift lambda(x) of the one-sided kernel on an axis [lo, hi] (reading R4):
+    the smallest |lambda| that keeps the support x + h [-(3k+1)/2 + lambda, (3k+1)/2 + lambda]
+    inside [lo, hi]; 0 in the interior (the symmetric kernel)."""
+    H = 0.5 * (3 * k + 1)
+    x = np.asarray(x, dtype=np.float64)
+    return np.maximum(0.0, H - (x - lo) / h) + np.minimum(0.0, (hi - x) / h - H)
+
+
+def kernel_values_shifted(k: int, c, lam: float, t) -> np.ndarray:
+    """K(t) = sum_g c_g psi(t - (g - k + lam)) from the C core (Cox-de Boor)."""
+    lib = _load()
+    t = np.ascontiguousarray(t, dtype=np.float64)
+    c = np.ascontiguousarray([float(v) for v in c], dtype=np.float64)
+    out = np.empty_like(t)
+    lib.oracle_kernel_shifted_many(k, _dp(c), float(lam), _dp(t), t.size, _dp(out))
+    return out
+
+
 def kernel_values(k: int, t) -> np.ndarray:
     """K(t) from the C core (Cox-de Boor) with the exact coefficients rounded to double."""
     lib = _load()
@@ -157,13 +203,17 @@ def gl_sizes(k: int, field_mode: int = 0, field_deg: int = 0) -> tuple[int, int]
 
 def oracle_eval(V, T, C, k: int, h: float, points, periodic: int = 3,
                 domain=(0.0, 0.0, 1.0, 1.0), field_mode: int = 0, field_deg: int = 0,
-                use_grid: bool | None = None, nthreads: int = 0, return_area: bool = False):
+                use_grid: bool | None = None, nthreads: int = 0, return_area: bool = False,
+                boundary: int = 0):
     """u*(x) at every point (Eq. (1)); see siac_oracle.c for the method.
 
     V (nv,2) f64; T (nt,3) int; C: (nt, (k+1)(k+2)/2) Dubiner modes (field_mode 0), the
     (d+1)^2 coefficients a[i, j] of y1^i y2^j (field_mode 1, d = field_deg), or (field_mode 2,
     the library's SIAC_BASIS_MONOMIAL_REF) per-triangle coefficients of r^a s^b on the unit
-    reference triangle (y = v0 + r (v1 - v0) + s (v2 - v0)), ordered by a + b, then b."""
+    reference triangle (y = v0 + r (v1 - v0) + s (v2 - v0)), ordered by a + b, then b.
+    boundary: 0 = zero extension on non-periodic axes; 1 = the one-sided kernel of ref [21] on
+    non-periodic axes (per point: lambda by onesided_shift, coefficients by
+    kernel_coefficients_shifted)."""
     lib = _load()
     V = np.ascontiguousarray(V, dtype=np.float64)
     T = np.ascontiguousarray(T, dtype=np.int32)
@@ -181,6 +231,24 @@ def oracle_eval(V, T, C, k: int, h: float, points, periodic: int = 3,
     gy, gwy = np.polynomial.legendre.leggauss(ny)
     out = np.zeros(len(P))
     area = np.zeros(len(P)) if return_area else None
+    pt_lam = pt_coef = None
+    if boundary == 1 and periodic != 3:
+        if (not periodic & 1 and W > dom[2] - dom[0] + 1e-12) or (not periodic & 2 and W > dom[3] - dom[1] + 1e-12):
+            raise ValueError("one-sided kernel: stencil width exceeds the domain")
+        pt_lam = np.zeros((len(P), 2))
+        for ax in (0, 1):
+            if not periodic & (1 << ax):
+                pt_lam[:, ax] = onesided_shift(k, h, P[:, ax], dom[ax], dom[ax + 2])
+        cache = {}
+        pt_coef = np.empty((len(P), 2, 2 * k + 1))
+        for i in range(len(P)):
+            for ax in (0, 1):
+                lv = float(pt_lam[i, ax])
+                if lv not in cache:
+                    cache[lv] = np.array([float(v) for v in kernel_coefficients_shifted(k, lv)])
+                pt_coef[i, ax] = cache[lv]
+        pt_lam = np.ascontiguousarray(pt_lam)
+        pt_coef = np.ascontiguousarray(pt_coef)
     if use_grid is None:
         use_grid = len(T) > 2000
     rc = lib.oracle_siac_eval(k, float(h), int(periodic), _dp(dom), _dp(V), len(V),
@@ -188,7 +256,9 @@ def oracle_eval(V, T, C, k: int, h: float, points, periodic: int = 3,
                               int(field_mode), _dp(C), int(field_deg), _dp(kc),
                               nx, _dp(gx), _dp(gwx), ny, _dp(gy), _dp(gwy),
                               _dp(P), len(P), _dp(out),
-                              _dp(area) if return_area else None, int(bool(use_grid)), int(nthreads))
+                              _dp(area) if return_area else None, int(bool(use_grid)), int(nthreads),
+                              _dp(pt_lam) if pt_lam is not None else None,
+                              _dp(pt_coef) if pt_coef is not None else None)
     if rc != 0:
         raise RuntimeError(f"oracle_siac_eval failed ({rc})")
     return (out, area) if return_area else out

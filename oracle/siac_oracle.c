@@ -63,6 +63,17 @@ double oracle_kernel(int k, const double *c, double t)
     return s;
 }
 
+/* The one-sided kernel of ref [21] (reading R4): the same 2k+1
+ * B-splines with every node shifted by lambda, x_g = -k + g + lambda, and coefficients c_g
+ * (supplied by oracle/__init__.py: the exact solution of the moment system at these nodes).
+ * lambda = 0 is the symmetric kernel. */
+double oracle_kernel_shifted(int k, const double *c, double lam, double t)
+{
+    double s = 0.0;
+    for (int g = 0; g <= 2 * k; ++g) s += c[g] * oracle_bspline(k, t - ((double)(g - k) + lam));
+    return s;
+}
+
 /* ------------------------------------------------------------------ Dubiner basis */
 
 /* Jacobi P_n^(alpha,0)(x) by the three-term recurrence (Abramowitz & Stegun 22.7.1). */
@@ -183,19 +194,21 @@ static int cmp_double(const void *a, const void *b)
 typedef struct { double m, q; } line;
 static inline double line_at(line L, double x) { return L.m * x + L.q; }
 
-/* Integral of K((y1-x1)/h) K((y2-x2)/h) u_t(y - s) over (T_t + s) for point x.
- * Adds the integral to *acc and the covered area to *area. */
+/* Integral of Kx((y1-x1)/h) Ky((y2-x2)/h) u_t(y - s) over (T_t + s) for point x, with
+ * Kx / Ky the kernels of coefficients kcx / kcy and node shifts lamx / lamy (0, P->kc: the
+ * symmetric kernel).  Adds the integral to *acc and the covered area to *area. */
 static void pair_integral(const problem *P, long t, double sx, double sy,
-                          double x1, double x2, nsum *acc, nsum *area)
+                          double x1, double x2, const double *kcx, const double *kcy,
+                          double lamx, double lamy, nsum *acc, nsum *area)
 {
     const int k = P->k;
     const double h = P->h;
-    const int nbr = 3 * k + 2;                /* breaklines t_m = -(3k+1)/2 + m, m = 0..3k+1 */
+    const int nbr = 3 * k + 2;                /* breaklines t_m = -(3k+1)/2 + lam + m, m = 0..3k+1 */
     double Xb[3 * MAXK + 2], Yb[3 * MAXK + 2];
     for (int m = 0; m < nbr; ++m) {
         double tm = -0.5 * (3 * k + 1) + m;
-        Xb[m] = x1 + h * tm;
-        Yb[m] = x2 + h * tm;
+        Xb[m] = x1 + h * (tm + lamx);
+        Yb[m] = x2 + h * (tm + lamy);
     }
     double px[3], py[3];
     for (int i = 0; i < 3; ++i) {
@@ -275,11 +288,11 @@ static void pair_integral(const problem *P, long t, double sx, double sy,
                 double wx = 0.5 * (b - a) * P->gwx[i];
                 double yg = line_at(g, x), yq = line_at(q, x);
                 double jy = 0.5 * (yq - yg);
-                double kx = oracle_kernel(k, P->kc, (x - x1) / h);
+                double kx = oracle_kernel_shifted(k, kcx, lamx, (x - x1) / h);
                 nadd(area, wx * 2.0 * jy);
                 for (int j = 0; j < P->ny; ++j) {
                     double y = yg + jy * (1.0 + P->gy[j]);
-                    double ky = oracle_kernel(k, P->kc, (y - x2) / h);
+                    double ky = oracle_kernel_shifted(k, kcy, lamy, (y - x2) / h);
                     double u = field_value(P, t, x - sx, y - sy);
                     nadd(acc, wx * jy * P->gwy[j] * kx * ky * u);
                 }
@@ -295,14 +308,17 @@ static void pair_integral(const problem *P, long t, double sx, double sy,
  * use_grid = 1: triangles are found through a bucket grid (each triangle is listed in every
  * bucket its bounding box touches; duplicates are skipped with a per-query stamp).
  * area_out (nullable): per point, the area of all integrated strips (the stencil area W^2
- * when the mesh covers the stencil).  Returns 0 on success. */
+ * when the mesh covers the stencil).
+ * pt_lam, pt_coef (nullable, the one-sided kernel): per point the node shifts (lambda_x,
+ * lambda_y) and the 2 x (2k+1) coefficients (x kernel, then y kernel); NULL = the symmetric
+ * kernel kc on both axes.  Returns 0 on success. */
 int oracle_siac_eval(int k, double h, int periodic, const double *domain,
                      const double *V, long nv, const int *T, long nt,
                      int field_mode, const double *field, int field_deg,
                      const double *kc, int nx, const double *gx, const double *gwx,
                      int ny, const double *gy, const double *gwy,
                      const double *pts, long np, double *out, double *area_out,
-                     int use_grid, int nthreads)
+                     int use_grid, int nthreads, const double *pt_lam, const double *pt_coef)
 {
     (void)nv;
     if (k < 1 || k > MAXK || nx > 64 || ny > 64) return -1;
@@ -366,16 +382,20 @@ int oracle_siac_eval(int k, double h, int periodic, const double *domain,
             if (periodic & 1) x1 = domain[0] + (x1 - domain[0]) - Lx * floor((x1 - domain[0]) / Lx);
             if (periodic & 2) x2 = domain[1] + (x2 - domain[1]) - Ly * floor((x2 - domain[1]) / Ly);
             nsum acc = {0, 0}, area = {0, 0};
+            const double lamx = pt_lam ? pt_lam[2 * p] : 0.0, lamy = pt_lam ? pt_lam[2 * p + 1] : 0.0;
+            const double *kcx = pt_coef ? pt_coef + (long)2 * (2 * k + 1) * p : kc;
+            const double *kcy = pt_coef ? kcx + (2 * k + 1) : kc;
             for (int si = -sxr; si <= sxr; ++si)
                 for (int sj = -syr; sj <= syr; ++sj) {
                     double sx = si * Lx, sy = sj * Ly;
-                    /* stencil box pulled back by the shift: images T+s meet the box iff T meets box-s */
-                    double qx0 = x1 - 0.5 * W - sx, qx1 = x1 + 0.5 * W - sx;
-                    double qy0 = x2 - 0.5 * W - sy, qy1 = x2 + 0.5 * W - sy;
+                    /* stencil box (moved by the node shift) pulled back by the image shift:
+                     * images T+s meet the box iff T meets box-s */
+                    double qx0 = x1 + h * lamx - 0.5 * W - sx, qx1 = x1 + h * lamx + 0.5 * W - sx;
+                    double qy0 = x2 + h * lamy - 0.5 * W - sy, qy1 = x2 + h * lamy + 0.5 * W - sy;
                     if (!use_grid) {
                         for (long t = 0; t < nt; ++t) {
                             if (bb[4 * t + 2] <= qx0 || bb[4 * t] >= qx1 || bb[4 * t + 3] <= qy0 || bb[4 * t + 1] >= qy1) continue;
-                            pair_integral(&P, t, sx, sy, x1, x2, &acc, &area);
+                            pair_integral(&P, t, sx, sy, x1, x2, kcx, kcy, lamx, lamy, &acc, &area);
                         }
                     } else {
                         ++query;
@@ -391,7 +411,7 @@ int oracle_siac_eval(int k, double h, int periodic, const double *domain,
                                     if (stamp[t] == query) continue;
                                     stamp[t] = query;
                                     if (bb[4 * t + 2] <= qx0 || bb[4 * t] >= qx1 || bb[4 * t + 3] <= qy0 || bb[4 * t + 1] >= qy1) continue;
-                                    pair_integral(&P, t, sx, sy, x1, x2, &acc, &area);
+                                    pair_integral(&P, t, sx, sy, x1, x2, kcx, kcy, lamx, lamy, &acc, &area);
                                 }
                             }
                     }
@@ -411,6 +431,11 @@ int oracle_siac_eval(int k, double h, int periodic, const double *domain,
 void oracle_kernel_many(int k, const double *c, const double *t, long n, double *out)
 {
     for (long i = 0; i < n; ++i) out[i] = oracle_kernel(k, c, t[i]);
+}
+
+void oracle_kernel_shifted_many(int k, const double *c, double lam, const double *t, long n, double *out)
+{
+    for (long i = 0; i < n; ++i) out[i] = oracle_kernel_shifted(k, c, lam, t[i]);
 }
 
 void oracle_bspline_many(int k, const double *t, long n, double *out)

@@ -125,18 +125,21 @@ def integrate_poly_triangle(p, A, B, C):
     return det * tot
 
 
-def exact_siac(V, T, fields, k, h, coeffs, x, periodic=3, L=(Fr(1), Fr(1))):
-    """u*(x) exactly.  V: list of (Fr, Fr); T: list of index triples; fields[t]: poly dict."""
+def exact_siac(V, T, fields, k, h, coeffs, x, periodic=3, L=(Fr(1), Fr(1)), coeffs_y=None):
+    """u*(x) exactly.  V: list of (Fr, Fr); T: list of index triples; fields[t]: poly dict.
+    coeffs_y: the y-axis kernel's coefficients if they differ from the x-axis' (one-sided
+    kernels, written on the symmetric node grid at the effective point)."""
     h = Fr(h)
     x1, x2 = Fr(x[0]), Fr(x[1])
     kp = kernel_cell_polys(k, coeffs)
+    kpy = kp if coeffs_y is None else kernel_cell_polys(k, coeffs_y)
     nc = 3 * k + 1
     tb = [Fr(-(3 * k + 1), 2) + i for i in range(nc + 1)]
     # K_i((y - x1)/h) as a polynomial in y1 (resp. y2)
     def kpoly_in(var, xc, i):
         lin = {(1, 0): 1 / h, (0, 0): -xc / h} if var == 0 else {(0, 1): 1 / h, (0, 0): -xc / h}
         out = {}
-        for m, c in enumerate(kp[i]):
+        for m, c in enumerate((kp if var == 0 else kpy)[i]):
             if c != 0:
                 out = padd(out, {mm: c * v for mm, v in ppow(lin, m).items()})
         return out
