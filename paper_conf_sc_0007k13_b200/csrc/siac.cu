@@ -39,6 +39,7 @@ struct siac_ctx {
     cudaStream_t stream = nullptr;   // the context's own non-blocking stream (create, siac_eval)
     int k = 1;
     int basis = 0, boundary = 0;
+    std::vector<double> os_pieces, os_ainv;   // one-sided kernel tables (siac::onesided_tables)
     siac_create_info cinfo = {};
     double h = 0, inv_h = 0;
     int periodic = 0;
@@ -294,6 +295,11 @@ void eval_device(siac_ctx *c, const double *d_pts, int64_t np, double *d_out, cu
     a.cw = c->cw; a.chh = c->chh; a.ex = c->ex; a.ey = c->ey;
     a.ncx = c->ncx; a.ncy = c->ncy; a.periodic = c->periodic;
     a.cnt = c->d_cnt;
+    a.os_axes = c->boundary == SIAC_BOUNDARY_ONESIDED ? (~c->periodic & 3) : 0;
+    a.x1d = c->dom[2]; a.y1d = c->dom[3];
+    a.os_pieces = c->os_pieces.data(); a.os_ainv = c->os_ainv.data();
+    need(a.os_axes == 0 || c->schedule == 0 || c->schedule == 5,
+         "SIAC_BOUNDARY_ONESIDED is implemented by the default schedule (JUMPX) only");
     if (c->counting) CK(cudaMemsetAsync(c->d_cnt, 0, 8 * sizeof(unsigned long long), st));
     cudaEvent_t ev_stop = nullptr;
     if (c->timing) {
@@ -413,7 +419,6 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
         if (p->boundary == SIAC_BOUNDARY_ONESIDED) {
             need((p->periodic & 1) || W <= Lx * (1 + 1e-12), "one-sided kernel: (3k+1)h exceeds the x-extent");
             need((p->periodic & 2) || W <= Ly * (1 + 1e-12), "one-sided kernel: (3k+1)h exceeds the y-extent");
-            need(p->periodic == 3, "SIAC_BOUNDARY_ONESIDED is not implemented yet");
         }
         need(nt <= (int64_t)0x3fffffff, "too many triangles");
         const int nb = (k + 1) * (k + 2) / 2;
@@ -452,6 +457,7 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
         CK(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
         c->basis = p->basis;
         c->boundary = p->boundary;
+        if (p->boundary == SIAC_BOUNDARY_ONESIDED) siac::onesided_tables(k, c->os_pieces, c->os_ainv);
         c->k = k;
         c->h = p->h;
         c->inv_h = 1.0 / p->h;

@@ -278,16 +278,18 @@ __device__ __forceinline__ void gen_pieces(const double *zx, const double *zy, E
 }
 
 // Contribution of one (point, triangle image) pair, integrated inline (thread-per-point
-// schedule).  kc: (3K+1) x (K+1) cell table.
+// schedule).  kc: (3K+1) x (K+1) cell table; kcy: the y axis' table if it differs (one-sided
+// kernels), else nullptr.
 template <int K, bool COUNT>
 __device__ double pair_contrib(const double *zx, const double *zy, const double *kc, const double *d,
-                               const PairGeom &g, Counts &cnt) {
+                               const PairGeom &g, Counts &cnt, const double *kcy = nullptr) {
+    if (kcy == nullptr) kcy = kc;
     constexpr double T0 = -0.5 * (3 * K + 1);
     double total = 0.0;
     auto emit = [&](const double *qx, const double *qy, int nq, int i, int j) {
         double kx[K + 1], ky[K + 1];
 #pragma unroll
-        for (int m = 0; m <= K; ++m) { kx[m] = kc[i * (K + 1) + m]; ky[m] = kc[j * (K + 1) + m]; }
+        for (int m = 0; m <= K; ++m) { kx[m] = kc[i * (K + 1) + m]; ky[m] = kcy[j * (K + 1) + m]; }
         if (COUNT) { cnt.pieces++; cnt.subtris += nq - 2; }
         for (int m = 1; m + 1 < nq; ++m)
             total += integrate_subtri<K>(qx[0], qy[0], qx[m], qy[m], qx[m + 1], qy[m + 1], kx, ky, T0 + i + 0.5,

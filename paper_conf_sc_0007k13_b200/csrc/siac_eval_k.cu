@@ -131,6 +131,19 @@ cudaError_t launch_part(const EvalArgs &a, bool count, int *, int num_sms, cudaS
     j.cell_start = a.cell_start; j.kc = a.kc; j.x0 = a.x0; j.y0 = a.y0; j.Lx = a.Lx; j.Ly = a.Ly;
     j.inv_h = a.inv_h; j.hw = a.hw; j.cw = a.cw; j.chh = a.chh; j.ex = a.ex; j.ey = a.ey;
     j.ncx = a.ncx; j.ncy = a.ncy; j.periodic = a.periodic; j.cnt = a.cnt;
+    // one-sided kernels near the non-periodic boundaries (schedule JUMPX only)
+    const bool os = a.os_axes != 0;
+    if (os && !a.xpoly) return cudaErrorInvalidValue;
+    j.os_axes = a.os_axes; j.h = a.h; j.x1d = a.x1d; j.y1d = a.y1d;
+    for (int i = 0; i < 25; ++i) j.osp[i] = 0.0;
+    for (int i = 0; i < 6; ++i) j.osb[i] = 0.0;
+    for (int i = 0; i < 81; ++i) j.osa[i] = 0.0;
+    if (os) {
+        for (int i = 0; i < (K + 1) * (K + 1); ++i) j.osp[i] = a.os_pieces[i];
+        for (int e = 0; e <= K + 1; ++e)      // beta_e = lead(piece e) - lead(piece e-1)
+            j.osb[e] = (e <= K ? a.os_pieces[e * (K + 1) + K] : 0.0) - (e >= 1 ? a.os_pieces[(e - 1) * (K + 1) + K] : 0.0);
+        for (int i = 0; i < (2 * K + 1) * (2 * K + 1); ++i) j.osa[i] = a.os_ainv[i];
+    }
     const int64_t ntiles = (a.np + 31) / 32;
     // fewer tiles than ~two waves of resident warps: split each tile's rows over 2 or 4 warps
     int split = 1;
@@ -139,15 +152,20 @@ cudaError_t launch_part(const EvalArgs &a, bool count, int *, int num_sms, cudaS
     const int tpb = siacjump::WARPS / split;
     const unsigned grid = (unsigned)((ntiles + tpb - 1) / tpb);
     const size_t smem = ((a.xpoly ? sizeof(siacjump::WarpSmemX) : sizeof(siacjump::WarpSmem)) +
-                         sizeof(siacjump::WarpStage<K>)) * siacjump::WARPS;
+                         sizeof(siacjump::WarpStage<K>) + (os ? sizeof(siacjump::OsSmem<K>) : 0)) * siacjump::WARPS;
     // GEN: some triangle is wider than h (in x or y), so a pair may see two knots on an axis
     const bool gen = std::max(a.ex, a.ey) > a.h * (1.0 + 1e-9);
-#define SIAC_LAUNCH_JUMP(C, G, XP)                                                                             \
+#define SIAC_LAUNCH_JUMP(C, G, XP, OS)                                                                         \
 do {                                                                                                           \
-    CK(cudaFuncSetAttribute(siacjump::k_eval_jump<K, C, G, XP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
-    siacjump::k_eval_jump<K, C, G, XP><<<grid, siacjump::WARPS * 32, smem, st>>>(j);                          \
+    CK(cudaFuncSetAttribute(siacjump::k_eval_jump<K, C, G, XP, OS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
+    siacjump::k_eval_jump<K, C, G, XP, OS><<<grid, siacjump::WARPS * 32, smem, st>>>(j);                      \
 } while (0)
-#define SIAC_LAUNCH_JUMP2(C, G) do { if (a.xpoly) SIAC_LAUNCH_JUMP(C, G, true); else SIAC_LAUNCH_JUMP(C, G, false); } while (0)
+#define SIAC_LAUNCH_JUMP2(C, G)                                                                                \
+do {                                                                                                           \
+    if (os) SIAC_LAUNCH_JUMP(C, G, true, true);                                                                \
+    else if (a.xpoly) SIAC_LAUNCH_JUMP(C, G, true, false);                                                     \
+    else SIAC_LAUNCH_JUMP(C, G, false, false);                                                                 \
+} while (0)
     if (count) { if (gen) SIAC_LAUNCH_JUMP2(true, true); else SIAC_LAUNCH_JUMP2(true, false); }
     else { if (gen) SIAC_LAUNCH_JUMP2(false, true); else SIAC_LAUNCH_JUMP2(false, false); }
 #undef SIAC_LAUNCH_JUMP2

@@ -27,6 +27,12 @@ struct EvalArgs {            // arguments of every evaluation schedule
     const int *pcell_start;   // schedule ELEM: point CSR by row-major binning cell
     int64_t nt;               // number of triangles
     unsigned long long *cnt;  // [candidates, pairs, pieces, subtris, corner, cross, cross_subtris, cross_polys]
+    // one-sided kernels (SIAC_BOUNDARY_ONESIDED; reading R4): axes (bit0 x, bit1 y)
+    // whose stencil shifts near the boundary, the domain's upper corner, and the host tables of
+    // siac::onesided_tables (B-spline pieces, inverse moment matrix) copied into the launch
+    int os_axes;
+    double x1d, y1d;
+    const double *os_pieces, *os_ainv;
 };
 
 // per (k, schedule part): p0 = jump, p1 = point, p2 = tile, p3 = warp-specialized

@@ -1,5 +1,6 @@
-// siac_jump.cuh -- schedule JUMP (the default): the exact decomposition of Eq. (2) reorganised
-// around the spline structure of the kernel, so that almost no per-pair quadrature is needed.
+// siac_jump.cuh -- schedules JUMPX (the default, SIAC_SCHEDULE_DEFAULT) and JUMP: the exact
+// decomposition of Eq. (2) reorganised around the spline structure of the kernel, so that almost
+// no per-pair quadrature is needed (JUMPX: none).
 //
 // Why it is exact.  K is a spline of degree k on the unit knots t_m = T0 + m (m = 0..3k+1,
 // T0 = -(3k+1)/2), C^{k-1} everywhere and zero outside [t_0, t_{3k+1}] (PAPER.md L196-208,
@@ -19,8 +20,10 @@
 //                                                lambda, so \int_{corner} (zeta1 - X)^k zeta2^b u
 //                                                = lambda^{k+2} G_b(lambda), G_b a polynomial of
 //                                                degree k+b precomputed per triangle at create time
-//     I11 = \int_{corner_x ∩ corner_y} C1 C2 u -- corner_x clipped by the line z2 = Y (SH), fan-
-//                                                triangulated, degree-3k Gauss quadrature.
+//     I11 = \int_{corner_x ∩ corner_y} C1 C2 u -- JUMP: corner_x clipped by the line z2 = Y (SH),
+//                                                fan-triangulated, degree-3k Gauss quadrature;
+//                                                JUMPX: a per-triangle interval polynomial in
+//                                                (lambda, Y') built at create time (§8.2b).
 // zeta = (y - centroid)/h is the per-triangle frame the precomputed data live in; z = zeta +
 // delta, delta = (centroid + image shift - x)/h.  Pairs with two or more knots inside a range
 // (only when h is smaller than the triangles) take the general per-pair path of siac_device.cuh.
@@ -347,16 +350,7 @@ __global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec) {
 #define SIAC_JUMP_PREFETCH 2      // candidates ahead whose hot record lines are prefetched into L1
 #endif
 constexpr int WARPS = SIAC_JUMP_WARPS;
-#ifndef SIAC_JUMP_LEAN
-#define SIAC_JUMP_LEAN 1          // 1: paired cell-table loads, one alpha read per pair (default; 0 = previous form)
-#endif
-#ifndef SIAC_JUMP_CSEL
-#define SIAC_JUMP_CSEL 0          // 1: corner coefficients by a third Taylor shift, not selects
-#endif
-#ifndef SIAC_JUMP_ILP2
-#define SIAC_JUMP_ILP2 0          // 1: two staged records evaluated per step (interleaved arithmetic)
-#endif
-constexpr int QCAP = SIAC_JUMP_ILP2 ? 96 : 64;   // cross-term queue: < 32 left over + 32 (64) new
+constexpr int QCAP = 64;      // cross-term queue: < 32 left over + <= 32 new
 constexpr int SCAP = 96;      // staged cross sub-triangles: < 32 left over + <= 64 new
 
 template <int SC> struct WarpSmemT {
@@ -392,6 +386,10 @@ template <int K> struct WarpStage {
     unsigned hm[32];          // their lane masks
 };
 
+template <int K> struct OsSmem {     // one-sided kernels: per-lane coefficients c[axis][g][lane]
+    double c[2][2 * K + 1][32];
+};
+
 struct JumpArgs {
     const double *pts;
     const int *perm;
@@ -409,6 +407,12 @@ struct JumpArgs {
     double cw, chh, ex, ey;
     int ncx, ncy, periodic;
     unsigned long long *cnt;  // candidates, pairs, pieces, subtris, corner, cross, cross_subtris, cross_polys
+    // one-sided kernels (template OS; reading R4): axes, h, the domain's upper corner,
+    // B-spline pieces (piece-major (K+1)^2), their leading-coefficient jumps beta_e (e = 0..K+1)
+    // and the inverse moment matrix ((2K+1)^2): c(lambda) = osa . (-lambda)^m
+    int os_axes;
+    double h, x1d, y1d;
+    double osp[25], osb[6], osa[81];
 };
 
 __device__ __forceinline__ double2 ld2(const double *p) { return __ldg(reinterpret_cast<const double2 *>(p)); }
@@ -498,23 +502,55 @@ __device__ __forceinline__ Cut axis_cut(const double *ad, double dd) {
 
 // Taylor coefficients p_a (a = 0..K) of the base cell polynomial at tau = zeta + e, in powers of
 // zeta.  kcp: padded cell table, row i+1 = cell i, rows 0 and NC+1 zero.
+template <int K> __device__ __forceinline__ void taylor_shift(double *p, double e) {
+#pragma unroll
+    for (int i = 0; i < K; ++i)
+#pragma unroll
+        for (int j = K - 1; j >= i; --j) p[j] = fma(e, p[j + 1], p[j]);
+}
 template <int K>
 __device__ __forceinline__ void base_taylor(const double *kcp, int row, double e, double *p) {
-#if SIAC_JUMP_LEAN
     if constexpr ((K & 1) == 1) {     // even row length: 16-byte aligned rows, paired loads
 #pragma unroll
         for (int j = 0; j <= K; j += 2) {
             const double2 t = *reinterpret_cast<const double2 *>(kcp + row * (K + 1) + j);
             p[j] = t.x; p[j + 1] = t.y;
         }
-    } else
-#endif
+    } else {
 #pragma unroll
-    for (int j = 0; j <= K; ++j) p[j] = kcp[row * (K + 1) + j];
+        for (int j = 0; j <= K; ++j) p[j] = kcp[row * (K + 1) + j];
+    }
+    taylor_shift<K>(p, e);
+}
+
+// One-sided kernels (SIAC_BOUNDARY_ONESIDED): the lane's kernel is Kt(t - lambda) with Kt on the
+// symmetric knot grid and coefficients c(lambda) (cl = &c[axis][0][lane], stride 32).  Row
+// `row` of its padded cell table (cell i = row - 1; rows 0 and NC+1 zero):
+//     Kt on cell i = sum_d c_{i-d} piece_d            (piece_d of psi_{k+1}, cell-centred)
+template <int K>
+__device__ __forceinline__ void os_row(const JumpArgs &a, const double *cl, int row, double *p) {
 #pragma unroll
-    for (int i = 0; i < K; ++i)
+    for (int j = 0; j <= K; ++j) p[j] = 0.0;
 #pragma unroll
-        for (int j = K - 1; j >= i; --j) p[j] = fma(e, p[j + 1], p[j]);
+    for (int d = 0; d <= K; ++d) {
+        const int g = row - 1 - d;
+        const bool ok = g >= 0 && g <= 2 * K;
+        const double cg = ok ? cl[(ok ? g : 0) * 32] : 0.0;
+#pragma unroll
+        for (int j = 0; j <= K; ++j) p[j] = fma(cg, a.osp[d * (K + 1) + j], p[j]);
+    }
+}
+// jump of Kt's leading coefficient across knot m: sum_e c_{m-e} beta_e
+template <int K>
+__device__ __forceinline__ double os_alpha(const JumpArgs &a, const double *cl, int m) {
+    double s = 0.0;
+#pragma unroll
+    for (int e = 0; e <= K + 1; ++e) {
+        const int g = m - e;
+        const bool ok = g >= 0 && g <= 2 * K;
+        s = fma(ok ? cl[(ok ? g : 0) * 32] : 0.0, a.osb[e], s);
+    }
+    return s;
 }
 
 // Estrin evaluation of sum_i c[i] x^i (N coefficients): dependency depth log2(N) instead of N.
@@ -598,7 +634,8 @@ struct GenOut {
 };
 template <int K, bool COUNT>
 __device__ __noinline__ GenOut general_pair(const double *__restrict__ rec, const double *kcp, int tri, double rsx,
-                                            double rsy, double x1, double x2, double inv_h) {
+                                            double rsy, double x1, double x2, double inv_h,
+                                            const double *kcpy = nullptr) {
     const double *rc = rec + (int64_t)Rec<K>::RS * tri;
     double zx[3], zy[3];
 #pragma unroll
@@ -614,7 +651,7 @@ __device__ __noinline__ GenOut general_pair(const double *__restrict__ rec, cons
     for (int m = 0; m < Rec<K>::NB; ++m) d[m] = __ldg(rc + Rec<K>::OFF_D + m);
     Counts cn = {0, 0, 0};
     GenOut o;
-    o.v = pair_contrib<K, COUNT>(zx, zy, kcp + (K + 1), d, g, cn);
+    o.v = pair_contrib<K, COUNT>(zx, zy, kcp + (K + 1), d, g, cn, kcpy ? kcpy + (K + 1) : nullptr);
     o.pieces = (unsigned)cn.pieces;
     o.subtris = (unsigned)cn.subtris;
     return o;
@@ -833,9 +870,10 @@ __device__ __forceinline__ double cross_I11(const double *jr, const double *xb, 
 
 // Closed-form cross terms of the top min(nq, 32) queue entries (one per lane), plus their
 // deferred y-corner terms, added to the owners' accumulators.
-template <int K, bool COUNT>
+template <int K, bool COUNT, bool OS = false>
 __device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, const double *kcp, const double *alpha,
-                                            int &nq, int lane, unsigned long long &c_poly) {
+                                            int &nq, int lane, unsigned long long &c_poly,
+                                            const OsSmem<K> *osm = nullptr) {
     using J = JRec<K>;
     using X = XRec<K>;
     const int take = min(nq, 32);
@@ -849,11 +887,20 @@ __device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, con
         const int sx = (info >> 5) & 1, sy = (info >> 6) & 1, mx = (info >> 7) & 31, my = (info >> 12) & 31;
         const int rowx = (info >> 17) & 31;
         const double *jr = a.jrec + (int64_t)J::RS * tri;
-        const double ay = sy == 0 ? alpha[my] : -alpha[my];
-        const double ax = sx == 0 ? alpha[mx] : -alpha[mx];
-        // deferred y-corner term of the pair
-        double pc[K + 1];
-        base_taylor<K>(kcp, rowx, S.qE[e], pc);
+        double ay, ax, pc[K + 1];
+        if constexpr (OS) {          // the owner lane's one-sided kernels
+            const int ol = info & 31;
+            const double amy = os_alpha<K>(a, &osm->c[1][0][ol], my);
+            const double amx = os_alpha<K>(a, &osm->c[0][0][ol], mx);
+            ay = sy == 0 ? amy : -amy;
+            ax = sx == 0 ? amx : -amx;
+            os_row<K>(a, &osm->c[0][0][ol], rowx, pc);
+            taylor_shift<K>(pc, S.qE[e]);
+        } else {
+            ay = sy == 0 ? alpha[my] : -alpha[my];
+            ax = sx == 0 ? alpha[mx] : -alpha[mx];
+            base_taylor<K>(kcp, rowx, S.qE[e], pc);       // (for the deferred y-corner term)
+        }
         const double ycorner = ay * corner_eval<K>(jr + J::OFF_G + (2 + sy) * J::NGP, pc, S.qL[e]);
         // the x corner's homothety ratio
         const double2 lh = ld2(jr + J::OFF_AX), iv = ld2(jr + J::OFF_AX + 4);
@@ -871,8 +918,12 @@ __device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, con
 #ifndef SIAC_JUMPX_MINB
 #define SIAC_JUMPX_MINB SIAC_JUMP_MINB
 #endif
-template <int K, bool COUNT, bool GEN, bool XP>
+// OS (one-sided kernels near non-periodic boundaries, with XP only): every lane evaluates its own
+// kernel Kt(. - lambda) at the effective point x + lambda h; cell rows and knot jumps are built
+// from the lane's coefficients (os_row / os_alpha) instead of the shared table.
+template <int K, bool COUNT, bool GEN, bool XP, bool OS = false>
 __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_MINB) k_eval_jump(JumpArgs a) {
+    static_assert(!OS || XP, "one-sided kernels are implemented for the closed-form cross terms (JUMPX)");
     using J = JRec<K>;
     constexpr int NC = 3 * K + 1;
     __shared__ __align__(16) double kcp[(NC + 2) * (K + 1)];
@@ -892,6 +943,8 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
     const int wid = threadIdx.x >> 5;
     WS &S = wsm[wid];
     WarpStage<K> &T = reinterpret_cast<WarpStage<K> *>(wsm + WARPS)[wid];
+    OsSmem<K> *osm = OS ? reinterpret_cast<OsSmem<K> *>(reinterpret_cast<WarpStage<K> *>(wsm + WARPS) + WARPS) + wid
+                        : nullptr;
     // a.split warps share one tile (small problems: more warps than tiles), each walking a
     // contiguous share of its candidate rows; partial sums are combined in a fixed order
     const int split = a.split;
@@ -916,6 +969,31 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
         x2 = a.pts[2 * (int64_t)orig + 1];
         if (a.periodic & 1) { x1 = x1 - a.Lx * floor((x1 - a.x0) / a.Lx); if (x1 >= a.x0 + a.Lx) x1 -= a.Lx; if (x1 < a.x0) x1 = a.x0; }
         if (a.periodic & 2) { x2 = x2 - a.Ly * floor((x2 - a.y0) / a.Ly); if (x2 >= a.y0 + a.Ly) x2 -= a.Ly; if (x2 < a.y0) x2 = a.y0; }
+    }
+    if constexpr (OS) {
+        // node shift lambda = the smallest |lambda| keeping x + h[-H + lambda, H + lambda] in the
+        // domain (0 in the interior); c(lambda) = osa . (-lambda)^m; then the effective point
+        constexpr double H = 0.5 * (3 * K + 1);
+        double lam[2] = {0.0, 0.0};
+        if (valid && (a.os_axes & 1)) lam[0] = fmax(0.0, H - (x1 - a.x0) / a.h) + fmin(0.0, (a.x1d - x1) / a.h - H);
+        if (valid && (a.os_axes & 2)) lam[1] = fmax(0.0, H - (x2 - a.y0) / a.h) + fmin(0.0, (a.y1d - x2) / a.h - H);
+#pragma unroll
+        for (int ax = 0; ax < 2; ++ax) {
+            double b[2 * K + 1];
+            b[0] = 1.0;
+#pragma unroll
+            for (int m = 1; m <= 2 * K; ++m) b[m] = -lam[ax] * b[m - 1];
+#pragma unroll
+            for (int g2 = 0; g2 <= 2 * K; ++g2) {
+                double c = 0.0;
+#pragma unroll
+                for (int m = 2 * K; m >= 0; --m) c = fma(a.osa[g2 * (2 * K + 1) + m], b[m], c);
+                osm->c[ax][g2][lane] = c;
+            }
+        }
+        x1 = fma(lam[0], a.h, x1);
+        x2 = fma(lam[1], a.h, x2);
+        __syncwarp();
     }
     S.acc[lane] = 0.0;
     double tx0 = valid ? x1 : 1e300, tx1 = valid ? x1 : -1e300, ty0 = valid ? x2 : 1e300, ty1 = valid ? x2 : -1e300;
@@ -952,7 +1030,7 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
     // then body(tri, rsx, rsy, hit, hr) for every candidate whose box meets the tile's stencils
     // (stg = true: only those some lane's stencil meets, hr = the record's hot part in shared
     // memory; else hr = nullptr).
-    auto candidates = [&](auto stg, auto &&body, auto &&body2) {
+    auto candidates = [&](auto stg, auto &&body) {
         for (int R = R0; R <= R1; ++R) {
             int r = R, qy = 0;
             if (a.periodic & 2) { r = ((R % a.ncy) + a.ncy) % a.ncy; qy = (R - r) / a.ncy; }
@@ -1003,30 +1081,6 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
                                 bulk_load(T.rec[sl], a.jrec + (int64_t)J::RS * (t_cur + T.hj[r]), HB, &T.bar[sl]);
                             }
                         }
-#if SIAC_JUMP_ILP2
-                        for (int i = 0; i < nh; i += 2) {
-                            const bool two = i + 1 < nh;                     // warp-uniform
-                            const int sa = (g + i) & (NST - 1), sb = (g + i + 1) & (NST - 1);
-                            mb_wait(&T.bar[sa], (ph >> sa) & 1u);
-                            ph ^= 1u << sa;
-                            if (two) {
-                                mb_wait(&T.bar[sb], (ph >> sb) & 1u);
-                                ph ^= 1u << sb;
-                            }
-                            const bool ha = ((T.hm[i] >> lane) & 1u) != 0;
-                            const bool hb = two && ((T.hm[i + 1] >> lane) & 1u) != 0;
-                            body2(t_cur + T.hj[i], ha, T.rec[sa], t_cur + T.hj[two ? i + 1 : i], hb,
-                                  T.rec[two ? sb : sa], rsx, rsy);
-                            __syncwarp();
-                            if (lane == 0) {
-                                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                                if (i + NST < nh)
-                                    bulk_load(T.rec[sa], a.jrec + (int64_t)J::RS * (t_cur + T.hj[i + NST]), HB, &T.bar[sa]);
-                                if (i + 1 + NST < nh)
-                                    bulk_load(T.rec[sb], a.jrec + (int64_t)J::RS * (t_cur + T.hj[i + 1 + NST]), HB, &T.bar[sb]);
-                            }
-                        }
-#else
                         for (int i = 0; i < nh; ++i) {
                             const int sl = (g + i) & (NST - 1);
                             mb_wait(&T.bar[sl], (ph >> sl) & 1u);
@@ -1038,7 +1092,6 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
                                 bulk_load(T.rec[sl], a.jrec + (int64_t)J::RS * (t_cur + T.hj[i + NST]), HB, &T.bar[sl]);
                             }
                         }
-#endif
                         g += nh;
                     } else {
                         for (int i = 0; i < nk; ++i) {
@@ -1073,8 +1126,15 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
             general = general || hit;     // integrated in the second pass below
         }
         double p[K + 1], q[K + 1];
-        base_taylor<K>(kcp, cx.row, cx.e, p);
-        base_taylor<K>(kcp, cy.row, cy.e, q);
+        if constexpr (OS) {
+            os_row<K>(a, &osm->c[0][0][lane], cx.row, p);
+            taylor_shift<K>(p, cx.e);
+            os_row<K>(a, &osm->c[1][0][lane], cy.row, q);
+            taylor_shift<K>(q, cy.e);
+        } else {
+            base_taylor<K>(kcp, cx.row, cx.e, p);
+            base_taylor<K>(kcp, cy.row, cy.e, q);
+        }
         double mu[J::NMU + 1];
 #pragma unroll
         for (int i = 0; i < J::NMU; i += 2) {
@@ -1095,25 +1155,16 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
         // both cut defers its y corner to the cross-term queue (clip_stage)
         const bool ux = cx.cut;
         const bool uy = !cx.cut && cy.cut;
-#if SIAC_JUMP_LEAN
         const int sdd = ux ? cx.side : cy.side;
-        const double am = alpha[ux ? cx.m : (uy ? cy.m : 0)];   // uncut: lam = 0 zeroes the corner
+        const int mm = ux ? cx.m : (uy ? cy.m : 0);              // uncut: lam = 0 zeroes the corner
+        double am;
+        if constexpr (OS) am = os_alpha<K>(a, &osm->c[ux ? 0 : 1][0][lane], mm);
+        else am = alpha[mm];
         const int sd = ux ? sdd : 2 + sdd;
         const double sg = sdd == 0 ? am : -am;
-#else
-        const double am = ux ? alpha[cx.m] : (uy ? alpha[cy.m] : 0.0);
-        const int sd = ux ? cx.side : 2 + cy.side;
-        const double sg = (ux ? cx.side : cy.side) == 0 ? am : -am;
-#endif
         double cc[K + 1];
-#if SIAC_JUMP_CSEL
-        // the other axis' Taylor coefficients, recomputed from selected (row, e) instead of
-        // K+1 double selects between p and q
-        base_taylor<K>(kcp, ux ? cy.row : cx.row, ux ? cy.e : cx.e, cc);
-#else
 #pragma unroll
         for (int j = 0; j <= K; ++j) cc[j] = ux ? q[j] : p[j];
-#endif
         const double lam = ux ? cx.lam : (uy ? cy.lam : 0.0);
         r.v = fma(sg, corner_eval<K, true>(hr + J::OFF_G + sd * J::NGP, cc, lam), v);
         r.cx = cx; r.cy = cy; r.skip = skip;
@@ -1143,7 +1194,7 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
     auto flush = [&]() {        // integrate queued cross terms 32 at a time (warp-uniform nq)
         while (nq >= 32) {
             if constexpr (XP) {
-                cross_stage<K, COUNT>(a, S, kcp, alpha, nq, lane, c_xpoly);
+                cross_stage<K, COUNT, OS>(a, S, kcp, alpha, nq, lane, c_xpoly, osm);
             } else {
                 clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
                 while (ns >= 32) integrate_stage<K>(a, S, alpha, ns, lane);
@@ -1154,18 +1205,9 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
         [&](int tri, double rsx, double rsy, bool hit, const double *hr) {
             pair_commit(tri, hit, pair_eval(rsx, rsy, hit, hr));
             flush();
-        },
-        // two staged records at once (SIAC_JUMP_ILP2): both evaluations are independent
-        // straight-line arithmetic the compiler interleaves; hb = false: B is a dummy (odd tail)
-        [&](int ta, bool ha, const double *ra, int tb, bool hb, const double *rb, double rsx, double rsy) {
-            const PairV va = pair_eval(rsx, rsy, ha, ra);
-            const PairV vb = pair_eval(rsx, rsy, hb, rb);
-            pair_commit(ta, ha, va);
-            pair_commit(tb, hb, vb);
-            flush();
         });
     if constexpr (XP) {
-        while (nq > 0) cross_stage<K, COUNT>(a, S, kcp, alpha, nq, lane, c_xpoly);
+        while (nq > 0) cross_stage<K, COUNT, OS>(a, S, kcp, alpha, nq, lane, c_xpoly, osm);
     } else {
         while (nq > 0) clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
         while (ns > 0) integrate_stage<K>(a, S, alpha, ns, lane);
@@ -1182,11 +1224,21 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
             const Cut cx = axis_cut<K, GEN>(jr + J::OFF_AX, fma((cen.x + rsx) - x1, a.inv_h, MT0));
             const Cut cy = axis_cut<K, GEN>(jr + J::OFF_AX + 6, fma((cen.y + rsy) - x2, a.inv_h, MT0));
             if (cx.multi || cy.multi) {
-                const GenOut go = general_pair<K, COUNT>(a.rec, kcp, tri, rsx, rsy, x1, x2, a.inv_h);
+                GenOut go;
+                if constexpr (OS) {        // the lane's two kernels as padded cell tables
+                    double tx[(NC + 2) * (K + 1)], ty[(NC + 2) * (K + 1)];
+                    for (int r = 0; r < NC + 2; ++r) {
+                        os_row<K>(a, &osm->c[0][0][lane], r, tx + r * (K + 1));
+                        os_row<K>(a, &osm->c[1][0][lane], r, ty + r * (K + 1));
+                    }
+                    go = general_pair<K, COUNT>(a.rec, tx, tri, rsx, rsy, x1, x2, a.inv_h, ty);
+                } else {
+                    go = general_pair<K, COUNT>(a.rec, kcp, tri, rsx, rsy, x1, x2, a.inv_h);
+                }
                 acc += go.v;
                 if (COUNT) { c_pieces += go.pieces; c_sub += go.subtris; }
             }
-        }, 0);
+        });
     }
     if (split == 1) {
         if (valid) a.out[orig] = acc + S.acc[lane];

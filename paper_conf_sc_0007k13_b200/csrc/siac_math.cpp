@@ -167,6 +167,50 @@ static std::vector<Q> kernel_coefficients_exact(int k) {
     return c;
 }
 
+// One-sided kernel support (SIAC_BOUNDARY_ONESIDED; reading R4).  The kernel with
+// nodes x_g = g - k + lambda is Kt(t - lambda), Kt on the symmetric node grid with moments
+// int Kt s^m = (-lambda)^m (m = 0..2k) -- expand (s + lambda)^m in the shifted kernel's
+// conditions int K t^m = delta_m0 -- so its coefficients are c(lambda) = A^{-1} b(lambda),
+// b_m = (-lambda)^m, with A the symmetric kernel's moment matrix.  Outputs (exact, rounded once):
+//   pieces[m*(k+1) + i]: psi_{k+1}'s piece m in the cell-centred variable (bspline_piece);
+//   ainv[g*(2k+1) + m]:  (A^{-1})_{g m}.
+void onesided_tables(int k, std::vector<double> &pieces, std::vector<double> &ainv) {
+    const int n = 2 * k + 1;
+    pieces.assign((size_t)(k + 1) * (k + 1), 0.0);
+    for (int m = 0; m <= k; ++m) {
+        P1 pc = bspline_piece(k, m);
+        for (int i = 0; i <= k; ++i) pieces[(size_t)m * (k + 1) + i] = pc[i].to_double();
+    }
+    std::vector<Q> mu(n);
+    for (int l = 0; l < n; ++l) mu[l] = bspline_moment(k, l);
+    std::vector<std::vector<Q>> A(n, std::vector<Q>(2 * n, Q(0)));
+    for (int m = 0; m < n; ++m) {
+        for (int g = 0; g < n; ++g) {
+            Q xg(g - k), s(0);
+            for (int l = 0; l <= m; ++l) s = s + Q(binom(m, l)) * qpow(xg, m - l) * mu[l];
+            A[m][g] = s;
+        }
+        A[m][n + m] = Q(1);
+    }
+    for (int col = 0; col < n; ++col) {
+        int piv = col;
+        while (piv < n && A[piv][col].zero()) ++piv;
+        if (piv == n) throw std::runtime_error("singular kernel moment system");
+        std::swap(A[col], A[piv]);
+        Q pv = A[col][col];
+        for (int j = col; j < 2 * n; ++j) A[col][j] = A[col][j] / pv;
+        for (int r = 0; r < n; ++r) {
+            if (r == col || A[r][col].zero()) continue;
+            Q f = A[r][col];
+            for (int j = col; j < 2 * n; ++j) A[r][j] = A[r][j] - f * A[col][j];
+        }
+    }
+    // rows of A now hold A^{-1} in columns n..2n-1: (A^{-1})_{g m} = A[g][n + m]
+    ainv.assign((size_t)n * n, 0.0);
+    for (int g = 0; g < n; ++g)
+        for (int m = 0; m < n; ++m) ainv[(size_t)g * n + m] = A[g][n + m].to_double();
+}
+
 // table[i*(k+1) + m]: coefficient of tau^m of K on cell i, tau = t - (t_i + 1/2).
 // On cell i, psi(t - x_g) is psi's piece i - g (when 0 <= i - g <= k), with the same local
 // variable (t_i - x_g = tau_{i-g}).

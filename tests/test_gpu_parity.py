@@ -434,3 +434,82 @@ def test_create_info(siac_mod):
     assert ci["total_ms"] >= ci["h2d_ms"] + ci["index_ms"] + ci["jump_ms"] + ci["cross_ms"]
     assert ci["bytes_per_triangle"] > 8 * inputs.n_modes(w.k)
     assert ci["device_bytes"] >= ci["bytes_per_triangle"] * len(w.T)
+
+
+# ------------------------------------------------------------------ one-sided kernels (NEXT-2)
+
+def _onesided_tol(oracle_mod, k, h, P, periodic, domain=(0.0, 0.0, 1.0, 1.0)):
+    """Per-point tolerance: north_star's 1e-10 relative, widened where the one-sided kernel's
+    coefficients are large (rounding ~ eps (sum|c_x|)(sum|c_y|); reading R4)."""
+    S = np.ones((len(P), 2))
+    for ax in (0, 1):
+        if not periodic & (1 << ax):
+            lam = oracle_mod.onesided_shift(k, h, P[:, ax], domain[ax], domain[ax + 2])
+            S[:, ax] = [sum(abs(float(c)) for c in oracle_mod.kernel_coefficients_shifted(k, float(l))) for l in lam]
+    return 1e-15 * S[:, 0] * S[:, 1]
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 4])
+@pytest.mark.parametrize("periodic", [0, 1, 2])
+def test_onesided_boundary_kernels(siac_mod, oracle_mod, k, periodic):
+    """SIAC_BOUNDARY_ONESIDED (ref [21]) on a non-periodic Delaunay mesh
+    covering the domain: every point, including boundary and corner points, against the
+    oracle's per-point shifted-node kernels."""
+    V, T = inputs.lattice_delaunay_mesh(3000, seed=50 + k)
+    C = inputs.random_modes(len(T), k, seed=60 + k)
+    h = inputs.max_edge(V, T)
+    P = inputs.eval_points(V, T, k)[::3]
+    P = np.concatenate([P, [[0, 0], [1, 1], [0, 1], [1, 0], [0.5, 0], [0, 0.5], [1, 0.3], [0.7, 1]]])
+    ctx = siac_mod.create(V, T, C, k, h, periodic=periodic, boundary=siac_mod.SIAC_BOUNDARY_ONESIDED)
+    g = ctx.eval(P)
+    ctx.destroy()
+    o = oracle_mod.oracle_eval(V, T, C, k, h, P, periodic=periodic, boundary=1)
+    tol = np.maximum(1e-10 * np.abs(o).max(), _onesided_tol(oracle_mod, k, h, P, periodic) * np.abs(o).max())
+    assert np.all(np.abs(g - o) <= tol), f"max excess {np.max(np.abs(g - o) / tol):.3e}"
+    assert_parity(g[np.abs(o) > 0], o[np.abs(o) > 0], tol=max(1e-10, float(_onesided_tol(oracle_mod, k, h, P, periodic).max())))
+
+
+@pytest.mark.parametrize("k", [1, 3])
+def test_onesided_reproduces_polynomials_to_the_boundary(siac_mod, k):
+    """A global polynomial of degree k is reproduced at every point up to the corners (the
+    one-sided kernel's purpose); zero extension is not (checked against the closed form)."""
+    V, T = inputs.lattice_delaunay_mesh(4000, seed=70 + k)
+    f = lambda x, y: 0.25 + (x - 0.4 * y) ** k - 0.6 * x * y ** (k - 1)  # noqa: E731
+    C = inputs.project(V, T, k, f)
+    h = inputs.max_edge(V, T)
+    P = np.concatenate([inputs.eval_points(V, T, k)[::5], [[0, 0], [1, 1], [0, 1], [1, 0]]])
+    ctx = siac_mod.create(V, T, C, k, h, periodic=0, boundary=siac_mod.SIAC_BOUNDARY_ONESIDED)
+    g = ctx.eval(P)
+    ctx.destroy()
+    assert np.abs(g - f(P[:, 0], P[:, 1])).max() < 1e-9
+    ctx = siac_mod.create(V, T, C, k, h, periodic=0)
+    gz = ctx.eval(P)
+    ctx.destroy()
+    assert np.abs(gz - f(P[:, 0], P[:, 1])).max() > 1e-3
+
+
+def test_onesided_small_h_general_path(siac_mod, oracle_mod):
+    """h smaller than the triangles (the clip-and-integrate pass inside the jump schedule) with
+    one-sided kernels on both axes."""
+    V, T = inputs.lattice_delaunay_mesh(1500, seed=77, graded=True)
+    k = 2
+    C = inputs.random_modes(len(T), k, seed=78)
+    h = 0.3 * inputs.max_edge(V, T)
+    P = np.concatenate([inputs.eval_points(V, T, k)[::11], [[0, 0], [1, 1], [0.02, 0.98]]])
+    ctx = siac_mod.create(V, T, C, k, h, periodic=0, boundary=1)
+    g = ctx.eval(P)
+    ctx.destroy()
+    o = oracle_mod.oracle_eval(V, T, C, k, h, P, periodic=0, boundary=1)
+    tol = np.maximum(1e-10, _onesided_tol(oracle_mod, k, h, P, 0)) * np.abs(o).max()
+    assert np.all(np.abs(g - o) <= tol)
+
+
+def test_onesided_rejects_other_schedules(siac_mod):
+    V, T = inputs.lattice_delaunay_mesh(500, seed=1)
+    C = inputs.random_modes(len(T), 1, seed=1)
+    ctx = siac_mod.create(V, T, C, 1, inputs.max_edge(V, T), periodic=0, boundary=1)
+    for sch in (1, 2, 3, 4, 6):
+        ctx.set_schedule(sch)
+        with pytest.raises(siac_mod.SiacError, match="one-sided|ONESIDED"):
+            ctx.eval(np.array([[0.5, 0.5]]))
+    ctx.destroy()
