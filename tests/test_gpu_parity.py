@@ -449,6 +449,24 @@ def _onesided_tol(oracle_mod, k, h, P, periodic, domain=(0.0, 0.0, 1.0, 1.0)):
     return 1e-15 * S[:, 0] * S[:, 1]
 
 
+def _onesided_sample(V, T, k, h, periodic, m=240):
+    """Element points: up to m inside the one-sided band of a non-periodic axis (every one has
+    its own lambda; the oracle solves its moment system exactly per point), m/2 interior ones,
+    plus the corners and edge midpoints."""
+    P = inputs.eval_points(V, T, k)
+    H = 0.5 * (3 * k + 1) * h
+    band = np.zeros(len(P), dtype=bool)
+    for ax in (0, 1):
+        if not periodic & (1 << ax):
+            band |= (P[:, ax] < H) | (P[:, ax] > 1 - H)
+    rng = np.random.default_rng(k + 10 * periodic)
+    bi, ii = np.nonzero(band)[0], np.nonzero(~band)[0]
+    pick = np.concatenate([rng.choice(bi, min(m, len(bi)), replace=False),
+                           rng.choice(ii, min(m // 2, len(ii)), replace=False)])
+    extra = np.array([[0, 0], [1, 1], [0, 1], [1, 0], [0.5, 0], [0, 0.5], [1, 0.3], [0.7, 1]])
+    return np.concatenate([P[np.sort(pick)], extra])
+
+
 @pytest.mark.parametrize("k", [1, 2, 3, 4])
 @pytest.mark.parametrize("periodic", [0, 1, 2])
 def test_onesided_boundary_kernels(siac_mod, oracle_mod, k, periodic):
@@ -458,8 +476,7 @@ def test_onesided_boundary_kernels(siac_mod, oracle_mod, k, periodic):
     V, T = inputs.lattice_delaunay_mesh(3000, seed=50 + k)
     C = inputs.random_modes(len(T), k, seed=60 + k)
     h = inputs.max_edge(V, T)
-    P = inputs.eval_points(V, T, k)[::3]
-    P = np.concatenate([P, [[0, 0], [1, 1], [0, 1], [1, 0], [0.5, 0], [0, 0.5], [1, 0.3], [0.7, 1]]])
+    P = _onesided_sample(V, T, k, h, periodic)
     ctx = siac_mod.create(V, T, C, k, h, periodic=periodic, boundary=siac_mod.SIAC_BOUNDARY_ONESIDED)
     g = ctx.eval(P)
     ctx.destroy()
@@ -495,7 +512,7 @@ def test_onesided_small_h_general_path(siac_mod, oracle_mod):
     k = 2
     C = inputs.random_modes(len(T), k, seed=78)
     h = 0.3 * inputs.max_edge(V, T)
-    P = np.concatenate([inputs.eval_points(V, T, k)[::11], [[0, 0], [1, 1], [0.02, 0.98]]])
+    P = _onesided_sample(V, T, k, h, 0, m=200)
     ctx = siac_mod.create(V, T, C, k, h, periodic=0, boundary=1)
     g = ctx.eval(P)
     ctx.destroy()
