@@ -269,10 +269,11 @@ siac_status siac_info(const siac_ctx *ctx, int64_t *n_triangles, int32_t *grid_n
  * Either pointer may be NULL. */
 siac_status siac_host_tables(int32_t k, double *cell_table, double *basis_matrix);
 
-/* Copy the first n device triangle records (record layout of csrc/siac_device.cuh, in
- * binning order) to host memory `out` (n * record_doubles); *record_doubles receives the
- * record length.  Diagnostics only. */
-siac_status siac_debug_records(siac_ctx *ctx, int64_t n, double *out, int32_t *record_doubles);
+/* Copy the first n device triangle records, in binning order, to host memory `out`
+ * (n * record_doubles); *record_doubles receives the record length.  which = 0: the mesh
+ * record (csrc/siac_device.cuh Rec), 1: the jump record (csrc/siac_jump.cuh JRec), 2: the
+ * closed-form cross-term record (XRec).  Diagnostics only. */
+siac_status siac_debug_records(siac_ctx *ctx, int32_t which, int64_t n, double *out, int32_t *record_doubles);
 
 /* Free everything the context owns.  NULL-safe. */
 void siac_destroy(siac_ctx *ctx);

@@ -804,16 +804,29 @@ siac_status siac_host_tables(int32_t k, double *cell_table, double *basis_matrix
     });
 }
 
-siac_status siac_debug_records(siac_ctx *ctx, int64_t n, double *out, int32_t *rd) {
+siac_status siac_debug_records(siac_ctx *ctx, int32_t which, int64_t n, double *out, int32_t *rd) {
     if (!ctx) { g_err = "NULL context"; return SIAC_EINVAL; }
     return run_guarded(&ctx->err, [&]() {
+        need(which >= 0 && which <= 2, "which must be 0, 1 or 2");
         const int nb = (ctx->k + 1) * (ctx->k + 2) / 2;
-        const int rs = (16 + nb + 1) & ~1;
+        int rs = (16 + nb + 1) & ~1;
+        const double *src = ctx->d_rec;
+        if (which == 1) {
+            static const int jrs[4] = {siacjump::JRec<1>::RS, siacjump::JRec<2>::RS, siacjump::JRec<3>::RS,
+                                       siacjump::JRec<4>::RS};
+            rs = jrs[ctx->k - 1];
+            src = ctx->d_jrec;
+        } else if (which == 2) {
+            const int xrs[4] = {siac_xrec_doubles_k1(), siac_xrec_doubles_k2(), siac_xrec_doubles_k3(),
+                                siac_xrec_doubles_k4()};
+            rs = xrs[ctx->k - 1];
+            src = ctx->d_xrec;
+        }
         if (rd) *rd = rs;
         need(n >= 0 && n <= ctx->nt, "n out of range");
         if (n > 0 && out) {
             CK(cudaSetDevice(ctx->device));
-            CK(cudaMemcpy(out, ctx->d_rec, sizeof(double) * rs * n, cudaMemcpyDeviceToHost));
+            CK(cudaMemcpy(out, src, sizeof(double) * rs * n, cudaMemcpyDeviceToHost));
         }
     });
 }

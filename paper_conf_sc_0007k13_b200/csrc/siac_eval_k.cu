@@ -5,6 +5,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cmath>
+#include <vector>
 
 #include "siac_device.cuh"
 #include "siac_internal.h"
@@ -242,8 +244,34 @@ cudaError_t SIAC_CAT(siac_prep_jump_k, SIAC_K)(const double *rec, int64_t nt, do
     siacjump::k_prep_jump<SIAC_K><<<(unsigned)((nt + 127) / 128), 128, 0, st>>>(rec, nt, h, jrec);
     return cudaGetLastError();
 }
+// Chebyshev interpolation -> monomial matrices (long double): for N nodes x_i = cos((2i+1)pi/2N),
+// the interpolant's Chebyshev coefficients are a_j = (w_j) sum_i f_i cos(j (2i+1) pi / 2N)
+// (w_0 = 1/N, else 2/N) and T_j = sum_m t_jm x^m (T_0 = 1, T_1 = x, T_j = 2x T_{j-1} - T_{j-2}),
+// so the coefficient of x^m is sum_i f_i sum_j t_jm w_j cos(j (2i+1) pi / 2N).
+static void cheb_mono_matrix(int N, double *mat, double *nodes) {
+    const long double pi = 3.141592653589793238462643383279502884L;
+    std::vector<long double> t((size_t)N * N, 0.0L);
+    t[0] = 1.0L;
+    if (N > 1) t[(size_t)1 * N + 1] = 1.0L;
+    for (int j = 2; j < N; ++j)
+        for (int m = 0; m < N; ++m)
+            t[(size_t)j * N + m] = (m > 0 ? 2.0L * t[(size_t)(j - 1) * N + m - 1] : 0.0L) - t[(size_t)(j - 2) * N + m];
+    for (int i = 0; i < N; ++i) nodes[i] = (double)cosl(pi * (2 * i + 1) / (2.0L * N));
+    for (int m = 0; m < N; ++m)
+        for (int i = 0; i < N; ++i) {
+            long double acc = 0.0L;
+            for (int j = m; j < N; ++j)
+                acc += t[(size_t)j * N + m] * (j == 0 ? 1.0L : 2.0L) / N * cosl(pi * j * (2 * i + 1) / (2.0L * N));
+            mat[(size_t)m * N + i] = (double)acc;
+        }
+}
+
 cudaError_t SIAC_CAT(siac_prep_cross_k, SIAC_K)(const double *jrec, int64_t nt, double *xrec, cudaStream_t st) {
-    siacjump::k_prep_cross<SIAC_K><<<(unsigned)((4 * nt + 127) / 128), 128, 0, st>>>(jrec, nt, xrec);
+    using X = siacjump::XRec<SIAC_K>;
+    siacjump::CrossTabs<SIAC_K> tb;
+    cheb_mono_matrix(X::NS, tb.ms, tb.node_s);
+    cheb_mono_matrix(X::NL, tb.ml, tb.node_l);
+    siacjump::k_prep_cross<SIAC_K><<<(unsigned)((4 * nt + 127) / 128), 128, 0, st>>>(jrec, nt, xrec, tb);
     return cudaGetLastError();
 }
 int SIAC_CAT(siac_xrec_doubles_k, SIAC_K)() { return siacjump::XRec<SIAC_K>::RS; }

@@ -51,6 +51,9 @@ using namespace siacdev;
 //   [OFF_MU ..]        mu[a*(K+1)+b] = \int_T zeta1^a zeta2^b u dzeta, a, b = 0..K (padded to even)
 //   [OFF_G ..]         4 corners (x-right, x-left, y-top, y-bottom) x NGP coefficients:
 //                      block b (= power of the other coordinate, 0..K) holds G_b[0..K+b]
+//   [OFF_XH ..]        per x corner side (0: apex R, 1: apex L): Ay, then the sorted heights
+//                      v0 <= v1 <= v2 of its reference corner (A, Mv, C') -- what the cross-term
+//                      classification needs at enqueue time (8 doubles)
 //   [OFF_GEO ..]       per axis: L, Mv, R (vertices sorted by that coordinate), C' (the point of
 //                      edge L-R at coordinate Mv) -- 8 doubles per axis
 //   [OFF_MAP ..]       rho = m00 z1 + m01 z2 + r0, sigma = m10 z1 + m11 z2 + s0 (centred reference
@@ -65,7 +68,8 @@ template <int K> struct JRec {
     static constexpr int OFF_AX = 2;
     static constexpr int OFF_MU = 14;
     static constexpr int OFF_G = OFF_MU + ((NMU + 1) & ~1);
-    static constexpr int OFF_GEO = OFF_G + 4 * NGP;
+    static constexpr int OFF_XH = OFF_G + 4 * NGP;
+    static constexpr int OFF_GEO = OFF_XH + 8;
     static constexpr int OFF_MAP = OFF_GEO + 16;
     static constexpr int OFF_D = OFF_MAP + 6;
     static constexpr int RAW = OFF_D + NB;
@@ -168,6 +172,17 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
         ad[5] = hi > mid ? 1.0 / (hi - mid) : 0.0;
         double *geo = o + J::OFF_GEO + 8 * ax;
         geo[0] = Lx; geo[1] = Ly; geo[2] = Mx; geo[3] = My; geo[4] = Rx; geo[5] = Ry; geo[6] = Cx; geo[7] = Cy;
+        if (ax == 0) {
+            for (int side = 0; side < 2; ++side) {   // heights of the reference corner (A, Mv, C')
+                const double Ay = side == 0 ? Ry : Ly;
+                double v[3] = {Ay, My, Cy};
+                if (v[0] > v[1]) { const double tt = v[0]; v[0] = v[1]; v[1] = tt; }
+                if (v[1] > v[2]) { const double tt = v[1]; v[1] = v[2]; v[2] = tt; }
+                if (v[0] > v[1]) { const double tt = v[0]; v[0] = v[1]; v[1] = tt; }
+                double *xh = o + J::OFF_XH + 4 * side;
+                xh[0] = Ay; xh[1] = v[0]; xh[2] = v[1]; xh[3] = v[2];
+            }
+        }
         for (int side = 0; side < 2; ++side) {      // 0: apex = R (right/top), 1: apex = L
             const double Ax = side == 0 ? Rx : Lx, Ay = side == 0 ? Ry : Ly;
             const double e1x = Mx - Ax, e1y = My - Ay, e2x = Cx - Ax, e2y = Cy - Ay;
@@ -210,10 +225,13 @@ __global__ void k_prep_jump(const double *rec, int64_t nt, double h, double *jre
 // z2 - Y = lambda (w2 - Y'), Y' = A2 + (Y - A2) / lambda, so
 //     I11 = lambda^{2K+2} F(lambda, Y'),  F = \int_{Cx ∩ H(Y')} (w1 - M1)^K (w2 - Y')^K u(A + lambda (w - A)) dw
 // over the fixed reference corner Cx = (A, M, C') clipped (Alg. 1) by the y knot line.  For the
-// half-plane above the line, F is a polynomial in (lambda, Y') of degree K x (3K + 2) on each of
-// the two intervals between the corner's vertex heights (the clipped region is a triangle with
-// vertices affine in Y'; the integrand has total degree 3K), 0 above the corner and the full-
-// corner integral below it (the corner polynomials G).  Below the line: full minus above.  The
+// half-plane above the line (y corner on the top side), F is a polynomial in (lambda, Y') of
+// degree K x (3K + 2) on each of the two intervals between the corner's vertex heights (the
+// clipped region is a triangle with vertices affine in Y'; the integrand has total degree 3K),
+// 0 above the corner and the full-corner integral below it (the corner polynomials G).  Below
+// the line (y corner on the bottom side) the same holds with "above" and "below" exchanged; its
+// interval polynomials F_below = F_full - F_above (F_full: the unclipped corner, degree K in
+// Y') are stored as well, so every in-interval cross term is ONE polynomial evaluation.  The
 // interval polynomials are built at create time by Chebyshev interpolation of exact samples
 // (each sample: SH clip of Cx + the degree-3K rule), stored as monomials in (mu, s) on
 // [-1, 1]^2 and evaluated column-wise in mu (independent short chains) then by Estrin in s.
@@ -222,8 +240,11 @@ template <int K> struct XRec {
     static constexpr int NL = K + 1;              // lambda degree + 1
     static constexpr int NLP = (NL + 1) & ~1;     // padded for 16-byte loads
     static constexpr int NP = NS * NLP;           // monomial coefficients m[j * NLP + i]: s^j mu^i
-    static constexpr int XB = (6 + 2 * NP + 1) & ~1;   // per x side: v0 v1 v2 iw0 iw1 0 | 2 x NP
+    // per x side: v0 v1 v2 iw0 iw1 0 | interval 0 above, interval 0 below, interval 1 above,
+    // interval 1 below (NP each)
+    static constexpr int XB = (6 + 4 * NP + 1) & ~1;
     static constexpr int RS = 2 * XB;
+    __host__ __device__ static constexpr int poly(int iv, int below) { return 6 + (2 * iv + below) * NP; }
 };
 
 // \int over triangle (p0, p1, p2) of (w1 - M1)^K (w2 - Yp)^K u(A + lam (w - A)), degree-3K rule;
@@ -247,9 +268,39 @@ __device__ double corner_piece(double p0x, double p0y, double p1x, double p1y, d
     return area * acc;
 }
 
-// One thread per (triangle, x side, interval): Chebyshev coefficients of F above the line.
+// Interpolation at Chebyshev nodes -> monomial coefficients, as two small matrices built on the
+// host in long double (siac_eval_k.cu): ms[jm * NS + is] maps the NS samples in s to the
+// coefficient of s^jm, ml[im * NL + il] the NL samples in lambda to the coefficient of mu^im
+// (mu = 2 lambda - 1); nodes cos((2i+1) pi / (2N)).  Passed by value (kernel parameters).
+template <int K> struct CrossTabs {
+    double ms[XRec<K>::NS * XRec<K>::NS];
+    double ml[XRec<K>::NL * XRec<K>::NL];
+    double node_s[XRec<K>::NS], node_l[XRec<K>::NL];
+};
+
+// (lambda, s) samples f[il][is] -> co[jm * NLP + im] (coefficient of s^jm mu^im), padding 0.
 template <int K>
-__global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec) {
+__device__ void samples_to_monomial(const CrossTabs<K> &tb, const double (*f)[XRec<K>::NS], double *co) {
+    using X = XRec<K>;
+    for (int jm = 0; jm < X::NS; ++jm) {
+        double g[X::NL];
+        for (int il = 0; il < X::NL; ++il) {
+            double acc = 0.0;
+            for (int is = 0; is < X::NS; ++is) acc = fma(tb.ms[jm * X::NS + is], f[il][is], acc);
+            g[il] = acc;
+        }
+        for (int im = 0; im < X::NLP; ++im) {
+            double acc = 0.0;
+            if (im < X::NL)
+                for (int il = 0; il < X::NL; ++il) acc = fma(tb.ml[im * X::NL + il], g[il], acc);
+            co[jm * X::NLP + im] = acc;
+        }
+    }
+}
+
+// One thread per (triangle, x side, interval): the above and below interval polynomials.
+template <int K>
+__global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec, const CrossTabs<K> tb) {
     using J = JRec<K>;
     using X = XRec<K>;
     const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -263,31 +314,29 @@ __global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec) {
     double mp[6], d[J::NB];
     for (int i = 0; i < 6; ++i) mp[i] = jr[J::OFF_MAP + i];
     for (int i = 0; i < J::NB; ++i) d[i] = jr[J::OFF_D + i];
-    double v[3] = {Ay, My, Cy};
-    if (v[0] > v[1]) { const double tt = v[0]; v[0] = v[1]; v[1] = tt; }
-    if (v[1] > v[2]) { const double tt = v[1]; v[1] = v[2]; v[2] = tt; }
-    if (v[0] > v[1]) { const double tt = v[0]; v[0] = v[1]; v[1] = tt; }
+    const double *xh = jr + J::OFF_XH + 4 * sx;     // sorted heights (k_prep_jump)
+    const double v0 = xh[1], v1 = xh[2], v2 = xh[3];
     double *xo = xrec + (int64_t)X::RS * t + sx * X::XB;
     if (iv == 0) {
-        xo[0] = v[0]; xo[1] = v[1]; xo[2] = v[2];
-        xo[3] = v[1] > v[0] ? 1.0 / (v[1] - v[0]) : 0.0;
-        xo[4] = v[2] > v[1] ? 1.0 / (v[2] - v[1]) : 0.0;
+        xo[0] = v0; xo[1] = v1; xo[2] = v2;
+        xo[3] = v1 > v0 ? 1.0 / (v1 - v0) : 0.0;
+        xo[4] = v2 > v1 ? 1.0 / (v2 - v1) : 0.0;
         xo[5] = 0.0;
-        for (int i = 6 + 2 * X::NP; i < X::XB; ++i) xo[i] = 0.0;
+        for (int i = 6 + 4 * X::NP; i < X::XB; ++i) xo[i] = 0.0;
     }
-    double *co = xo + 6 + iv * X::NP;
-    const double a = v[iv], b = v[iv + 1];
+    double *ca = xo + X::poly(iv, 0), *cb = xo + X::poly(iv, 1);
+    const double a = iv == 0 ? v0 : v1, b = iv == 0 ? v1 : v2;
     if (!(b > a)) {
-        for (int i = 0; i < X::NP; ++i) co[i] = 0.0;
+        for (int i = 0; i < X::NP; ++i) { ca[i] = 0.0; cb[i] = 0.0; }
         return;
     }
-    double f[X::NL][X::NS];
+    double fa[X::NL][X::NS], fb[X::NL][X::NS];
+    const double px[3] = {Ax, Mx, Cx}, py[3] = {Ay, My, Cy};
     for (int il = 0; il < X::NL; ++il) {
-        const double lam = 0.5 * (cospi((2.0 * il + 1.0) / (2.0 * X::NL)) + 1.0);
+        const double lam = 0.5 * (tb.node_l[il] + 1.0);
         for (int is = 0; is < X::NS; ++is) {
-            const double Yp = a + 0.5 * (cospi((2.0 * is + 1.0) / (2.0 * X::NS)) + 1.0) * (b - a);
+            const double Yp = a + 0.5 * (tb.node_s[is] + 1.0) * (b - a);
             // Sutherland-Hodgman clip of (A, M, C') by w2 >= Yp, fan from the first vertex
-            const double px[3] = {Ax, Mx, Cx}, py[3] = {Ay, My, Cy};
             double qx[4], qy[4];
             int n = 0;
             for (int e = 0; e < 3; ++e) {
@@ -302,40 +351,14 @@ __global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec) {
             double F = 0.0;
             for (int j = 1; j + 1 < n; ++j)
                 F += corner_piece<K>(qx[0], qy[0], qx[j], qy[j], qx[j + 1], qy[j + 1], Mx, Yp, Ax, Ay, lam, mp, d);
-            f[il][is] = F;
+            // the whole corner at the same (lambda, Y'): F_below = F_full - F_above
+            const double Ffull = corner_piece<K>(Ax, Ay, Mx, My, Cx, Cy, Mx, Yp, Ax, Ay, lam, mp, d);
+            fa[il][is] = F;
+            fb[il][is] = Ffull - F;
         }
     }
-    // discrete Chebyshev transform in Y' (s) then in lambda (mu)
-    double c1[X::NL][X::NS];
-    for (int il = 0; il < X::NL; ++il)
-        for (int j = 0; j < X::NS; ++j) {
-            double acc = 0.0;
-            for (int is = 0; is < X::NS; ++is) acc += f[il][is] * cospi((double)(j * (2 * is + 1)) / (2.0 * X::NS));
-            c1[il][j] = acc * ((j == 0 ? 1.0 : 2.0) / X::NS);
-        }
-    double c2[X::NL][X::NS];
-    for (int i = 0; i < X::NL; ++i)
-        for (int j = 0; j < X::NS; ++j) {
-            double acc = 0.0;
-            for (int il = 0; il < X::NL; ++il) acc += c1[il][j] * cospi((double)(i * (2 * il + 1)) / (2.0 * X::NL));
-            c2[i][j] = acc * ((i == 0 ? 1.0 : 2.0) / X::NL);
-        }
-    // Chebyshev -> monomial in both variables (T_j coefficients by the integer recurrence)
-    double tc[X::NS][X::NS];
-    for (int j = 0; j < X::NS; ++j)
-        for (int k = 0; k < X::NS; ++k) tc[j][k] = 0.0;
-    tc[0][0] = 1.0;
-    if (X::NS > 1) tc[1][1] = 1.0;
-    for (int j = 2; j < X::NS; ++j)
-        for (int k = 0; k < X::NS; ++k) tc[j][k] = (k > 0 ? 2.0 * tc[j - 1][k - 1] : 0.0) - tc[j - 2][k];
-    for (int jm = 0; jm < X::NS; ++jm)
-        for (int im = 0; im < X::NLP; ++im) {
-            double acc = 0.0;
-            if (im < X::NL)
-                for (int i = im; i < X::NL; ++i)
-                    for (int j = jm; j < X::NS; ++j) acc += tc[i][im] * tc[j][jm] * c2[i][j];
-            co[jm * X::NLP + im] = acc;
-        }
+    samples_to_monomial<K>(tb, fa, ca);
+    samples_to_monomial<K>(tb, fb, cb);
 }
 
 // ------------------------------------------------------------------ evaluation
@@ -368,7 +391,25 @@ template <int SC> struct WarpSmemT {
     int klist[32];            // kept candidates of the current chunk (box meets the tile's stencils)
 };
 using WarpSmem = WarpSmemT<SCAP>;     // schedule JUMP: staged cross sub-triangles
-using WarpSmemX = WarpSmemT<2>;       // schedule JUMPX: no sub-triangles (smaller)
+
+// Schedule JUMPX: cross terms classified at enqueue time (while the record is staged) into two
+// queues that are each evaluated 32 at a time without divergence:
+//   qp  "poly":  the y knot line cuts the x corner -> one interval polynomial (above / below);
+//   qf  "full":  the line misses it -> the whole-corner integral (corner polynomials) or 0.
+// Every entry also carries the pair's deferred y-corner term.
+struct XQueue {
+    int tri[QCAP];
+    int info[QCAP];           // lane | sx << 6 | sy << 7 | mx << 8 | my << 13 | row_x << 18 | iv << 23 | full << 24
+    double Y[QCAP];           // y knot (zeta frame of the triangle)
+    double E[QCAP], L[QCAP];  // deferred y-corner term: base-x offset e_x, y homothety ratio
+    double lam[QCAP];         // x corner homothety ratio
+};
+struct WarpSmemX {
+    XQueue qp, qf;
+    double acc[32];
+    double4 cbox[32];
+    int klist[32];
+};
 template <bool XP> using WarpSmemFor = typename std::conditional<XP, WarpSmemX, WarpSmem>::type;
 
 #ifndef SIAC_JUMP_STAGES
@@ -823,57 +864,71 @@ __device__ __forceinline__ double mono2d(const double *m, double mu, double s) {
     return estrin<NS>(col, s);
 }
 
-// I11 / (sgn alpha_x sgn alpha_y): \int_{x corner ∩ y corner} (z1 - X)^K (z2 - Y)^K u for the x
-// corner of side sx with homothety ratio lam, the y knot Y (zeta frame) and the y corner on side
+// Binomial coefficients of (zeta2 - Y)^K in powers of zeta2: cy[b] = C(K, b) (-Y)^(K-b).
+template <int K> __device__ __forceinline__ void ypow_coeffs(double Y, double *cy) {
+    double pw = 1.0;
+#pragma unroll
+    for (int b = K; b >= 0; --b) {
+        double bin = 1.0;
+#pragma unroll
+        for (int r = 0; r < K - b; ++r) bin = bin * (double)(K - r) / (double)(r + 1);
+        cy[b] = bin * pw;
+        pw *= -Y;
+    }
+}
+
+// lambda^{2K+2} F_dir(lambda, Y') on interval iv of the x corner of side sx: the y knot Y' in
+// the reference corner's frame, s its position in the interval, dir = sy (0 above, 1 below).
+template <int K>
+__device__ __forceinline__ double cross_poly(const double *xb, double Ay, double lam, double Y, int iv, int dir) {
+    using X = XRec<K>;
+    const double Yp = fma(Y - Ay, 1.0 / lam, Ay);
+    const double va = __ldg(xb + iv), iw = __ldg(xb + 3 + iv);
+    const double sv = fma(2.0 * (Yp - va), iw, -1.0);
+    double l2k = lam * lam;
+#pragma unroll
+    for (int i = 0; i < K; ++i) l2k *= lam * lam;
+    return l2k * mono2d<X::NL, X::NLP, X::NS>(xb + X::poly(iv, dir), 2.0 * lam - 1.0, sv);
+}
+
+// Classification of a cross term (the y knot Y against the x corner of side sx, homothety lam):
+// 0 = the line misses the corner on the far side (I11 = 0), 1 = it misses it on the near side
+// (I11 = the whole corner), 2 = it cuts interval 0, 3 = it cuts interval 1.  xh: the record's
+// (Ay, v0, v1, v2) of that side; the test Y' <> v is written as (Y - Ay) <> lam (v - Ay), lam > 0.
+__device__ __forceinline__ int cross_class(const double *xh, double lam, double Y, int sy) {
+    const double d = Y - xh[0];
+    const bool below_all = d <= lam * (xh[1] - xh[0]);      // Y' <= v0: the line under the corner
+    const bool above_all = d >= lam * (xh[3] - xh[0]);      // Y' >= v2
+    if (!below_all && !above_all) return d < lam * (xh[2] - xh[0]) ? 2 : 3;
+    return (sy == 0 ? below_all : above_all) ? 1 : 0;
+}
+
+// I11 / (sgn alpha_x sgn alpha_y) of one pair, evaluated inline (per-element schedule): the
+// x corner of side sx with homothety ratio lam, the y knot Y (zeta frame), the y corner on side
 // sy; xb = the triangle's XRec block of side sx.  poly: evaluated by an interval polynomial.
 template <int K>
 __device__ __forceinline__ double cross_I11(const double *jr, const double *xb, double lam, double Y, int sx, int sy,
                                             bool &poly) {
     using J = JRec<K>;
-    using X = XRec<K>;
-    const double Ay = __ldg(jr + J::OFF_GEO + (sx == 0 ? 5 : 1));
-    const double2 v01 = ld2(xb), v2i = ld2(xb + 2), i1 = ld2(xb + 4);
-    const double Yp = fma(Y - Ay, 1.0 / lam, Ay);     // the y knot in the reference corner's frame
-    const bool above_all = Yp >= v2i.x;                // the line is above the corner
-    const bool below_all = Yp <= v01.x;                // ... below it
-    // the full-corner integral of (z1 - X)^K (z2 - Y)^K u: corner polynomials with the
-    // coefficients of (zeta2 - Y)^K in powers of zeta2
-    const bool need_full = sy == 0 ? below_all : !below_all;
-    double full = 0.0;
-    if (need_full) {
-        double cy[K + 1];
-        double pw = 1.0;
+    double xh[4];
 #pragma unroll
-        for (int b = K; b >= 0; --b) {      // C(K, b) (-Y)^{K-b}
-            double bin = 1.0;
-#pragma unroll
-            for (int r = 0; r < K - b; ++r) bin = bin * (double)(K - r) / (double)(r + 1);
-            cy[b] = bin * pw;
-            pw *= -Y;
-        }
-        full = corner_eval<K>(jr + J::OFF_G + sx * J::NGP, cy, lam);
-    }
-    double part = 0.0;                                 // lambda^{2K+2} F_above(lambda, Y')
-    const bool inside = !above_all && !below_all;
-    if (inside) {
-        const bool lo = Yp < v01.y;
-        const double va = lo ? v01.x : v01.y, iw = lo ? v2i.y : i1.x;
-        const double sv = fma(2.0 * (Yp - va), iw, -1.0);
-        double l2k = lam * lam;
-#pragma unroll
-        for (int i = 0; i < K; ++i) l2k *= lam * lam;
-        part = l2k * mono2d<X::NL, X::NLP, X::NS>(xb + 6 + (lo ? 0 : X::NP), 2.0 * lam - 1.0, sv);
-    }
-    poly = inside;
-    return sy == 0 ? (inside ? part : (below_all ? full : 0.0)) : (inside ? full - part : (above_all ? full : 0.0));
+    for (int i = 0; i < 4; ++i) xh[i] = __ldg(jr + J::OFF_XH + 4 * sx + i);
+    const int cls = cross_class(xh, lam, Y, sy);
+    poly = cls >= 2;
+    if (cls >= 2) return cross_poly<K>(xb, xh[0], lam, Y, cls - 2, sy);
+    if (cls == 0) return 0.0;
+    double cy[K + 1];
+    ypow_coeffs<K>(Y, cy);
+    return corner_eval<K>(jr + J::OFF_G + sx * J::NGP, cy, lam);
 }
 
-// Closed-form cross terms of the top min(nq, 32) queue entries (one per lane), plus their
-// deferred y-corner terms, added to the owners' accumulators.
-template <int K, bool COUNT, bool OS = false>
-__device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, const double *kcp, const double *alpha,
-                                            int &nq, int lane, unsigned long long &c_poly,
-                                            const OsSmem<K> *osm = nullptr) {
+// Evaluate the top min(nq, 32) entries of queue Q (one per lane): the deferred y-corner term
+// plus sgn alpha_x sgn alpha_y I11, POLY = true: interval polynomials (qp), else whole corner
+// or 0 (qf); added to the owners' accumulators.
+template <int K, bool COUNT, bool OS, bool POLY>
+__device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, XQueue &Q, const double *kcp,
+                                            const double *alpha, int &nq, int lane, unsigned long long &c_poly,
+                                            const OsSmem<K> *osm) {
     using J = JRec<K>;
     using X = XRec<K>;
     const int take = min(nq, 32);
@@ -881,11 +936,11 @@ __device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, con
     double val = 0.0;
     if (lane < take) {
         const int e = nq - 1 - lane;
-        const int tri = S.qtri[e], info = S.qinfo[e];
-        const double Xk = S.qX[e], Y = S.qY[e];
-        key = info & 31;
-        const int sx = (info >> 5) & 1, sy = (info >> 6) & 1, mx = (info >> 7) & 31, my = (info >> 12) & 31;
-        const int rowx = (info >> 17) & 31;
+        const int tri = Q.tri[e], info = Q.info[e];
+        const double Y = Q.Y[e], lam = Q.lam[e];
+        key = info & 63;
+        const int sx = (info >> 6) & 1, sy = (info >> 7) & 1, mx = (info >> 8) & 31, my = (info >> 13) & 31;
+        const int rowx = (info >> 18) & 31, iv = (info >> 23) & 1, full = (info >> 24) & 1;
         const double *jr = a.jrec + (int64_t)J::RS * tri;
         double ay, ax, pc[K + 1];
         if constexpr (OS) {          // the owner lane's one-sided kernels
@@ -895,19 +950,23 @@ __device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, con
             ay = sy == 0 ? amy : -amy;
             ax = sx == 0 ? amx : -amx;
             os_row<K>(a, &osm->c[0][0][ol], rowx, pc);
-            taylor_shift<K>(pc, S.qE[e]);
+            taylor_shift<K>(pc, Q.E[e]);
         } else {
             ay = sy == 0 ? alpha[my] : -alpha[my];
             ax = sx == 0 ? alpha[mx] : -alpha[mx];
-            base_taylor<K>(kcp, rowx, S.qE[e], pc);       // (for the deferred y-corner term)
+            base_taylor<K>(kcp, rowx, Q.E[e], pc);       // (for the deferred y-corner term)
         }
-        const double ycorner = ay * corner_eval<K>(jr + J::OFF_G + (2 + sy) * J::NGP, pc, S.qL[e]);
-        // the x corner's homothety ratio
-        const double2 lh = ld2(jr + J::OFF_AX), iv = ld2(jr + J::OFF_AX + 4);
-        const double lam = sx == 0 ? (lh.y - Xk) * iv.y : (Xk - lh.x) * iv.x;
-        bool poly = false;
-        const double I11 = cross_I11<K>(jr, a.xrec + (int64_t)X::RS * tri + sx * X::XB, lam, Y, sx, sy, poly);
-        if (COUNT && poly) ++c_poly;
+        const double ycorner = ay * corner_eval<K>(jr + J::OFF_G + (2 + sy) * J::NGP, pc, Q.L[e]);
+        double I11 = 0.0;
+        if constexpr (POLY) {
+            const double Ay = __ldg(jr + J::OFF_XH + 4 * sx);
+            I11 = cross_poly<K>(a.xrec + (int64_t)X::RS * tri + sx * X::XB, Ay, lam, Y, iv, sy);
+            if (COUNT) ++c_poly;
+        } else if (full) {
+            double cy[K + 1];
+            ypow_coeffs<K>(Y, cy);
+            I11 = corner_eval<K>(jr + J::OFF_G + sx * J::NGP, cy, lam);
+        }
         val = fma(ax * ay, I11, ycorner);
     }
     nq -= take;
@@ -1020,7 +1079,8 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
     __syncwarp();
 
     double acc = 0.0;
-    int nq = 0, ns = 0;
+    int nq = 0, ns = 0;       // JUMP: cross-term queue, staged sub-triangles
+    int nqp = 0, nqf = 0;     // JUMPX: poly / full cross-term queues
     bool general = false;     // this lane met a pair with several knots on an axis
 
     unsigned long long c_cand = 0, c_pairs = 0, c_pieces = 0, c_sub = 0, c_corner = 0, c_cross = 0, c_xsub = 0,
@@ -1170,13 +1230,43 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
         r.cx = cx; r.cy = cy; r.skip = skip;
         return r;
     };
-    auto pair_commit = [&](int tri, bool hit, const PairV &r) {
+    auto pair_commit = [&](int tri, bool hit, const PairV &r, const double *hr) {
         const Cut &cx = r.cx, &cy = r.cy;
         if (hit && !r.skip) acc += r.v;
         const bool cross = hit && !r.skip && cx.cut && cy.cut;
         if (COUNT && hit && !r.skip) c_corner += (int)cx.cut + (int)cy.cut;
         const unsigned cm = __ballot_sync(0xffffffffu, cross);
-        if (cm) {
+        if constexpr (XP) {
+            // classify each cross term against its x corner's heights (staged record) and
+            // append it to the poly or the full queue
+            if (cm) {
+                int cls = 0;
+                if (cross) {
+                    const double2 h01 = ldr2<true>(hr + J::OFF_XH + 4 * cx.side);
+                    const double2 h23 = ldr2<true>(hr + J::OFF_XH + 4 * cx.side + 2);
+                    const double xh[4] = {h01.x, h01.y, h23.x, h23.y};
+                    cls = cross_class(xh, cx.lam, cy.X, cy.side);
+                }
+                const bool isp = cross && cls >= 2;
+                const unsigned pm = __ballot_sync(0xffffffffu, isp);
+                const unsigned fm = cm & ~pm;
+                if (cross) {
+                    XQueue &Q = isp ? S.qp : S.qf;
+                    const int pos = isp ? nqp + __popc(pm & lanemask_lt()) : nqf + __popc(fm & lanemask_lt());
+                    Q.tri[pos] = tri;
+                    Q.info[pos] = lane | (cx.side << 6) | (cy.side << 7) | (cx.m << 8) | (cy.m << 13) | (cx.row << 18) |
+                                  ((cls == 3) << 23) | ((cls == 1) << 24);
+                    Q.Y[pos] = cy.X;
+                    Q.E[pos] = cx.e;
+                    Q.L[pos] = cy.lam;
+                    Q.lam[pos] = cx.lam;
+                }
+                nqp += __popc(pm);
+                nqf += __popc(fm);
+                if (COUNT) c_cross += __popc(cm) * (lane == 0);
+                __syncwarp();
+            }
+        } else if (cm) {
             if (cross) {
                 const int pos = nq + __popc(cm & lanemask_lt());
                 S.qtri[pos] = tri;
@@ -1191,11 +1281,12 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
             __syncwarp();
         }
     };
-    auto flush = [&]() {        // integrate queued cross terms 32 at a time (warp-uniform nq)
-        while (nq >= 32) {
-            if constexpr (XP) {
-                cross_stage<K, COUNT, OS>(a, S, kcp, alpha, nq, lane, c_xpoly, osm);
-            } else {
+    auto flush = [&]() {        // evaluate queued cross terms 32 at a time (warp-uniform counts)
+        if constexpr (XP) {
+            while (nqp >= 32) cross_stage<K, COUNT, OS, true>(a, S, S.qp, kcp, alpha, nqp, lane, c_xpoly, osm);
+            while (nqf >= 32) cross_stage<K, COUNT, OS, false>(a, S, S.qf, kcp, alpha, nqf, lane, c_xpoly, osm);
+        } else {
+            while (nq >= 32) {
                 clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
                 while (ns >= 32) integrate_stage<K>(a, S, alpha, ns, lane);
             }
@@ -1203,11 +1294,12 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
     };
     candidates(std::true_type{},
         [&](int tri, double rsx, double rsy, bool hit, const double *hr) {
-            pair_commit(tri, hit, pair_eval(rsx, rsy, hit, hr));
+            pair_commit(tri, hit, pair_eval(rsx, rsy, hit, hr), hr);
             flush();
         });
     if constexpr (XP) {
-        while (nq > 0) cross_stage<K, COUNT, OS>(a, S, kcp, alpha, nq, lane, c_xpoly, osm);
+        while (nqp > 0) cross_stage<K, COUNT, OS, true>(a, S, S.qp, kcp, alpha, nqp, lane, c_xpoly, osm);
+        while (nqf > 0) cross_stage<K, COUNT, OS, false>(a, S, S.qf, kcp, alpha, nqf, lane, c_xpoly, osm);
     } else {
         while (nq > 0) clip_stage<K, COUNT>(a, S, kcp, alpha, nq, ns, lane, c_xsub);
         while (ns > 0) integrate_stage<K>(a, S, alpha, ns, lane);

@@ -162,7 +162,7 @@ def lib():
         L.siac_host_tables.restype = ctypes.c_int
         L.siac_host_tables.argtypes = [I32, D, D]
         L.siac_debug_records.restype = ctypes.c_int
-        L.siac_debug_records.argtypes = [vp, I64, D, ctypes.POINTER(I32)]
+        L.siac_debug_records.argtypes = [vp, I32, I64, D, ctypes.POINTER(I32)]
         L.siac_destroy.restype = None
         L.siac_destroy.argtypes = [vp]
         L.siac_last_error.restype = ctypes.c_char_p
@@ -301,11 +301,12 @@ class Context:
                                ctypes.byref(cw), ctypes.byref(ch)), self._ptr)
         return dict(n_triangles=nt.value, grid_nx=gx.value, grid_ny=gy.value, cell_w=cw.value, cell_h=ch.value)
 
-    def debug_records(self, n: int) -> np.ndarray:
+    def debug_records(self, n: int, which: int = 0) -> np.ndarray:
+        """First n device records in binning order: which = 0 mesh (Rec), 1 jump (JRec), 2 cross (XRec)."""
         rd = ctypes.c_int32()
-        _check(lib().siac_debug_records(self._ptr, 0, None, ctypes.byref(rd)), self._ptr)
+        _check(lib().siac_debug_records(self._ptr, int(which), 0, None, ctypes.byref(rd)), self._ptr)
         out = np.empty((n, rd.value))
-        _check(lib().siac_debug_records(self._ptr, n, _dp(out), ctypes.byref(rd)), self._ptr)
+        _check(lib().siac_debug_records(self._ptr, int(which), n, _dp(out), ctypes.byref(rd)), self._ptr)
         return out
 
     def destroy(self) -> None:
