@@ -107,8 +107,9 @@ struct Fail {
             throw Fail{SIAC_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_)};        \
     } while (0)
 
-inline void need(bool ok, const std::string &msg) {
-    if (!ok) throw Fail{SIAC_EINVAL, msg};
+// (const char *: the hot validation loops must not build a std::string per check)
+inline void need(bool ok, const char *msg) {
+    if (__builtin_expect(!ok, 0)) throw Fail{SIAC_EINVAL, std::string(msg)};
 }
 
 // ------------------------------------------------------------------ create kernels
@@ -447,9 +448,14 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
         int ndev = 0;
         if (cudaGetDeviceCount(&ndev) != cudaSuccess || p->device < 0 || p->device >= ndev)
             throw Fail{SIAC_EDEVICE, "no CUDA device with that ordinal"};
-        cudaDeviceProp prop;
-        CK(cudaGetDeviceProperties(&prop, p->device));
-        if (prop.major < 10) throw Fail{SIAC_EDEVICE, std::string("device is not sm_100 class: ") + prop.name};
+        int major = 0, nsm = 0;
+        CK(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, p->device));
+        CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device));
+        if (major < 10) {
+            cudaDeviceProp prop;
+            CK(cudaGetDeviceProperties(&prop, p->device));
+            throw Fail{SIAC_EDEVICE, std::string("device is not sm_100 class: ") + prop.name};
+        }
         CK(cudaSetDevice(p->device));
 
         c = new siac_ctx();
@@ -484,7 +490,7 @@ siac_status siac_create(siac_ctx **out, const double *V, int64_t nv, const int32
         CK(cudaMemcpy(c->d_kc, kc.data(), sizeof(double) * kc.size(), cudaMemcpyHostToDevice));
         CK(cudaMalloc(&c->d_cnt, 8 * sizeof(unsigned long long)));
         CK(cudaMalloc(&c->d_tile_counter, sizeof(int)));
-        c->num_sms = prop.multiProcessorCount;
+        c->num_sms = nsm;
         CK(cudaMemsetAsync(c->d_cnt, 0, 8 * sizeof(unsigned long long), c->stream));
         const int64_t ncell = (int64_t)c->ncx * c->ncy;
         CK(cudaMalloc(&c->d_cell_start, sizeof(int) * (ncell + 1)));
