@@ -34,10 +34,13 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
 
+_SRC3 = os.path.join(_HERE, "siac_oracle3d.c")
+
+
 def build_oracle(force: bool = False) -> str:
-    """Compile siac_oracle.c -> oracle/liboracle.so (gcc -O2 -fopenmp)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-o", _LIB, _SRC, "-lm"])
+    """Compile siac_oracle.c + siac_oracle3d.c -> oracle/liboracle.so (gcc -O2 -fopenmp)."""
+    if force or not os.path.exists(_LIB) or any(os.path.getmtime(_LIB) < os.path.getmtime(f) for f in (_SRC, _SRC3)):
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-o", _LIB, _SRC, _SRC3, "-lm"])
     return _LIB
 
 
@@ -52,6 +55,9 @@ def _load():
                                          I, D, I, D, I, D, D, I, D, D, D, L, D, D, I, I, D, D]
         lib.oracle_kernel_many.argtypes = [I, D, D, L, D]
         lib.oracle_kernel_shifted_many.argtypes = [I, D, ctypes.c_double, D, L, D]
+        lib.oracle_siac_eval3.restype = I
+        lib.oracle_siac_eval3.argtypes = [I, ctypes.c_double, I, D, D, L, ctypes.POINTER(ctypes.c_int), L,
+                                          I, D, I, D, I, D, D, D, L, D, D, I]
         lib.oracle_bspline_many.argtypes = [I, D, L, D]
         lib.oracle_dubiner_many.argtypes = [I, D, D, L, D]
         _lib = lib
@@ -270,3 +276,47 @@ def omp_threads() -> int:
         return len(os.sched_getaffinity(0))
     except AttributeError:  # pragma: no cover
         return os.cpu_count() or 1
+
+
+# ----------------------------------------------------------------------------- 3D (NEXT-4)
+
+def n_modes3(k: int) -> int:
+    return (k + 1) * (k + 2) * (k + 3) // 6
+
+
+def oracle_eval3(V, T, C, k: int, h: float, points, periodic: int = 7,
+                 domain=(0.0, 0.0, 0.0, 1.0, 1.0, 1.0), field_mode: int = 0, field_deg: int = 0,
+                 nthreads: int = 0, return_volume: bool = False):
+    """u*(x) on a tetrahedral mesh (the 3D form of Eq. (1); siac_oracle3d.c for the method).
+
+    V (nv,3); T (nt,4) int; C: (nt, n_modes3(k)) coefficients of r^a s^b t^c on the unit
+    reference tetrahedron (y = v0 + r (v1-v0) + s (v2-v0) + t (v3-v0); modes by n = a+b+c, then
+    c, then b) for field_mode 0, or (d+1)^3 coefficients a[i, j, l] of y1^i y2^j y3^l
+    (field_mode 1, d = field_deg).  periodic: bit d = axis d."""
+    lib = _load()
+    V = np.ascontiguousarray(V, dtype=np.float64)
+    T = np.ascontiguousarray(T, dtype=np.int32)
+    C = np.ascontiguousarray(C, dtype=np.float64)
+    P = np.ascontiguousarray(points, dtype=np.float64).reshape(-1, 3)
+    dom = np.ascontiguousarray(domain, dtype=np.float64)
+    W = (3 * k + 1) * h
+    for d in range(3):
+        if periodic & (1 << d) and W > dom[d + 3] - dom[d] + 1e-12:
+            raise ValueError("stencil width exceeds a periodic extent")
+    kc = np.array([float(v) for v in kernel_coefficients(k)])
+    # degree of the x-integrand K(x) S(x) between breakpoints: K_x (k) times the section integral
+    # of K_y K_z u (total degree 2k + k for dG, 2k + 3d for x^i y^j z^l) over a polygon whose
+    # vertices move linearly in x (+2); the y- and z-integrands have lower degree.  An n-point
+    # Gauss rule is exact to degree 2n-1.
+    deg = (k + 3 * k if field_mode == 0 else 3 * k + 3 * field_deg) + 2
+    n = deg // 2 + 1
+    g, w = np.polynomial.legendre.leggauss(n)
+    out = np.zeros(len(P))
+    vol = np.zeros(len(P)) if return_volume else None
+    rc = lib.oracle_siac_eval3(k, float(h), int(periodic), _dp(dom), _dp(V), len(V),
+                               T.ctypes.data_as(ctypes.POINTER(ctypes.c_int)), len(T), int(field_mode), _dp(C),
+                               int(field_deg), _dp(kc), n, _dp(g), _dp(w), _dp(P), len(P), _dp(out),
+                               _dp(vol) if return_volume else None, int(nthreads))
+    if rc != 0:
+        raise RuntimeError(f"oracle_siac_eval3 failed ({rc})")
+    return (out, vol) if return_volume else out

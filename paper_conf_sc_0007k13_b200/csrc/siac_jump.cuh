@@ -427,8 +427,8 @@ template <int K> struct WarpStage {
     unsigned hm[32];          // their lane masks
 };
 
-template <int K> struct OsSmem {     // one-sided kernels: per-lane coefficients c[axis][g][lane]
-    double c[2][2 * K + 1][32];
+template <int K, int NPT = 32> struct OsSmem {   // one-sided kernels: per-point c[axis][g][point]
+    double c[2][2 * K + 1][NPT];
 };
 
 struct JumpArgs {
@@ -504,10 +504,9 @@ struct Cut {
 // within rounding of each end: either choice drops a sliver that is empty to rounding).  The
 // base cell is the one below the knot when the knot is above the middle vertex (corner on the
 // high side), else the one above; with no knot inside, the cell holding the range.
-template <int K, bool GEN, bool SM = false>
-__device__ __forceinline__ Cut axis_cut(const double *ad, double dd) {
+template <int K, bool GEN>
+__device__ __forceinline__ Cut axis_cut_r(double2 lh, double2 mz, double2 iv, double dd) {
     constexpr int NC = 3 * K + 1;
-    const double2 lh = ldr2<SM>(ad), mz = ldr2<SM>(ad + 2), iv = ldr2<SM>(ad + 4);
     const double lo = lh.x + dd, hi = lh.y + dd;
     Cut c;
     c.multi = false;
@@ -540,6 +539,11 @@ __device__ __forceinline__ Cut axis_cut(const double *ad, double dd) {
     c.lam = hs ? (hi - mk) * iv.y : (mk - lo) * iv.x;
     return c;
 }
+// the axis data (lo, hi | mid, c5 | invL, invR) read from ad (shared memory if SM)
+template <int K, bool GEN, bool SM = false>
+__device__ __forceinline__ Cut axis_cut(const double *ad, double dd) {
+    return axis_cut_r<K, GEN>(ldr2<SM>(ad), ldr2<SM>(ad + 2), ldr2<SM>(ad + 4), dd);
+}
 
 // Taylor coefficients p_a (a = 0..K) of the base cell polynomial at tau = zeta + e, in powers of
 // zeta.  kcp: padded cell table, row i+1 = cell i, rows 0 and NC+1 zero.
@@ -568,7 +572,7 @@ __device__ __forceinline__ void base_taylor(const double *kcp, int row, double e
 // symmetric knot grid and coefficients c(lambda) (cl = &c[axis][0][lane], stride 32).  Row
 // `row` of its padded cell table (cell i = row - 1; rows 0 and NC+1 zero):
 //     Kt on cell i = sum_d c_{i-d} piece_d            (piece_d of psi_{k+1}, cell-centred)
-template <int K>
+template <int K, int NPT = 32>
 __device__ __forceinline__ void os_row(const JumpArgs &a, const double *cl, int row, double *p) {
 #pragma unroll
     for (int j = 0; j <= K; ++j) p[j] = 0.0;
@@ -576,20 +580,20 @@ __device__ __forceinline__ void os_row(const JumpArgs &a, const double *cl, int 
     for (int d = 0; d <= K; ++d) {
         const int g = row - 1 - d;
         const bool ok = g >= 0 && g <= 2 * K;
-        const double cg = ok ? cl[(ok ? g : 0) * 32] : 0.0;
+        const double cg = ok ? cl[(ok ? g : 0) * NPT] : 0.0;
 #pragma unroll
         for (int j = 0; j <= K; ++j) p[j] = fma(cg, a.osp[d * (K + 1) + j], p[j]);
     }
 }
 // jump of Kt's leading coefficient across knot m: sum_e c_{m-e} beta_e
-template <int K>
+template <int K, int NPT = 32>
 __device__ __forceinline__ double os_alpha(const JumpArgs &a, const double *cl, int m) {
     double s = 0.0;
 #pragma unroll
     for (int e = 0; e <= K + 1; ++e) {
         const int g = m - e;
         const bool ok = g >= 0 && g <= 2 * K;
-        s = fma(ok ? cl[(ok ? g : 0) * 32] : 0.0, a.osb[e], s);
+        s = fma(ok ? cl[(ok ? g : 0) * NPT] : 0.0, a.osb[e], s);
     }
     return s;
 }
@@ -727,7 +731,7 @@ __device__ __forceinline__ void seg_add(SM_ &S, int key, double v, int lane) {
         const double w = __shfl_sync(0xffffffffu, v, src);
         if (rest) { if (lane == leader) sum += w; rest &= rest - 1; }
     }
-    if (lane == leader && key < 32) S.acc[key] += sum;
+    if (lane == leader && key < (int)(sizeof(S.acc) / sizeof(S.acc[0]))) S.acc[key] += sum;
     __syncwarp();
 }
 
@@ -925,14 +929,14 @@ __device__ __forceinline__ double cross_I11(const double *jr, const double *xb, 
 // Evaluate the top min(nq, 32) entries of queue Q (one per lane): the deferred y-corner term
 // plus sgn alpha_x sgn alpha_y I11, POLY = true: interval polynomials (qp), else whole corner
 // or 0 (qf); added to the owners' accumulators.
-template <int K, bool COUNT, bool OS, bool POLY>
-__device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, XQueue &Q, const double *kcp,
+template <int K, bool COUNT, bool OS, bool POLY, class SM_, int NPT = 32>
+__device__ __forceinline__ void cross_stage(const JumpArgs &a, SM_ &S, XQueue &Q, const double *kcp,
                                             const double *alpha, int &nq, int lane, unsigned long long &c_poly,
-                                            const OsSmem<K> *osm) {
+                                            const OsSmem<K, NPT> *osm) {
     using J = JRec<K>;
     using X = XRec<K>;
     const int take = min(nq, 32);
-    int key = 32 + lane;
+    int key = NPT + lane;                       // (>= the number of points: ignored by seg_add)
     double val = 0.0;
     if (lane < take) {
         const int e = nq - 1 - lane;
@@ -943,13 +947,13 @@ __device__ __forceinline__ void cross_stage(const JumpArgs &a, WarpSmemX &S, XQu
         const int rowx = (info >> 18) & 31, iv = (info >> 23) & 1, full = (info >> 24) & 1;
         const double *jr = a.jrec + (int64_t)J::RS * tri;
         double ay, ax, pc[K + 1];
-        if constexpr (OS) {          // the owner lane's one-sided kernels
-            const int ol = info & 31;
-            const double amy = os_alpha<K>(a, &osm->c[1][0][ol], my);
-            const double amx = os_alpha<K>(a, &osm->c[0][0][ol], mx);
+        if constexpr (OS) {          // the owner point's one-sided kernels
+            const int ol = info & 63;
+            const double amy = os_alpha<K, NPT>(a, &osm->c[1][0][ol], my);
+            const double amx = os_alpha<K, NPT>(a, &osm->c[0][0][ol], mx);
             ay = sy == 0 ? amy : -amy;
             ax = sx == 0 ? amx : -amx;
-            os_row<K>(a, &osm->c[0][0][ol], rowx, pc);
+            os_row<K, NPT>(a, &osm->c[0][0][ol], rowx, pc);
             taylor_shift<K>(pc, Q.E[e]);
         } else {
             ay = sy == 0 ? alpha[my] : -alpha[my];

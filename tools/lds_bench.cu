@@ -32,9 +32,21 @@ __global__ void __launch_bounds__(128) k_lds(double *out, int iters) {
             } else if (MODE == 4) { // 1 x 128-bit, 2 distinct addresses
                 const double2 v = *reinterpret_cast<const double2 *>(buf + ((off & 511) + 22 * (lane & 1)));
                 acc0 += v.x; acc1 += v.y;
-            } else {                // 1 x 128-bit, 13 distinct rows of 4 doubles (lane % 13)
+            } else if (MODE == 5) { // 1 x 128-bit, 13 distinct rows of 4 doubles (lane % 13)
                 const double2 v = *reinterpret_cast<const double2 *>(buf + ((off & 511) + 4 * (lane % 13)));
                 acc0 += v.x; acc1 += v.y;
+            } else if (MODE == 6) { // 4 distinct contiguous 16 B chunks (lane & 3)
+                const double2 v = *reinterpret_cast<const double2 *>(buf + ((off & 511) + 2 * (lane & 3)));
+                acc0 += v.x; acc1 += v.y;
+            } else if (MODE == 7) { // 13 distinct contiguous 16 B chunks (lane % 13)
+                const double2 v = *reinterpret_cast<const double2 *>(buf + ((off & 511) + 2 * (lane % 13)));
+                acc0 += v.x; acc1 += v.y;
+            } else if (MODE == 8) { // 4 distinct chunks, 4 per half-warp-contiguous pattern: (lane >> 3)
+                const double2 v = *reinterpret_cast<const double2 *>(buf + ((off & 511) + 2 * (lane >> 3)));
+                acc0 += v.x; acc1 += v.y;
+            } else {                // 64-bit loads, 13 distinct contiguous doubles (lane % 13)
+                acc0 += buf[(off & 511) + (lane % 13)];
+                acc1 += buf[(off & 511) + 16 + (lane % 13)];
             }
         }
         base += 2;
@@ -49,9 +61,10 @@ int main() {
     cudaEvent_t e0, e1;
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);
-    const char *names[6] = {"4x LDS.32 uniform", "2x LDS.64 uniform", "1x LDS.128 uniform", "1x LDS.128 4 addrs",
-                            "1x LDS.128 2 addrs", "1x LDS.128 13 rows"};
-    for (int m = 0; m < 6; ++m) {
+    const char *names[10] = {"4x LDS.32 uniform", "2x LDS.64 uniform", "1x LDS.128 uniform", "1x LDS.128 4 addrs",
+                             "1x LDS.128 2 addrs", "1x LDS.128 13 rows", "128 4 contiguous", "128 13 contiguous",
+                             "128 4 contig lane>>3", "2x LDS.64 13 contig"};
+    for (int m = 0; m < 10; ++m) {
         for (int rep = 0; rep < 2; ++rep) {
             cudaEventRecord(e0);
             if (m == 0) k_lds<0><<<grid, 128>>>(d, iters);
@@ -60,6 +73,10 @@ int main() {
             if (m == 3) k_lds<3><<<grid, 128>>>(d, iters);
             if (m == 4) k_lds<4><<<grid, 128>>>(d, iters);
             if (m == 5) k_lds<5><<<grid, 128>>>(d, iters);
+            if (m == 6) k_lds<6><<<grid, 128>>>(d, iters);
+            if (m == 7) k_lds<7><<<grid, 128>>>(d, iters);
+            if (m == 8) k_lds<8><<<grid, 128>>>(d, iters);
+            if (m == 9) k_lds<9><<<grid, 128>>>(d, iters);
             cudaEventRecord(e1);
             cudaEventSynchronize(e1);
         }
