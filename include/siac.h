@@ -275,6 +275,45 @@ siac_status siac_host_tables(int32_t k, double *cell_table, double *basis_matrix
  * closed-form cross-term record (XRec).  Diagnostics only. */
 siac_status siac_debug_records(siac_ctx *ctx, int32_t which, int64_t n, double *out, int32_t *record_doubles);
 
+/* ---- Tetrahedral meshes ("extension of these ideas to
+ * 3D over unstructured tetrahedral meshes").  The 3D form of Eq. (1) -- the stencil is the tensor
+ * product of three 1D kernels (L212-214) -- integrated exactly as in Eq. (2): each tetrahedron
+ * the stencil touches is cut by the kernel breakplanes into pieces inside single kernel cells
+ * (depth-first plane splits; a cut tetrahedron is a tetrahedron + a prism or two prisms, a prism
+ * 3 tetrahedra), each piece integrated by a collapsed Gauss-Jacobi rule exact for degree 3k.
+ * Direct method (thread per point); conventions as for the 2D calls above. */
+typedef struct siac3_ctx siac3_ctx;
+typedef struct {
+    int32_t k;          /* dG degree 1..3 */
+    double  h;          /* kernel scaling > 0 */
+    int32_t periodic;   /* bit d (0..2): axis d periodic; non-periodic axes use zero extension */
+    double  domain[6];  /* x0, y0, z0, x1, y1, z1 */
+    int32_t device;
+} siac3_params;
+
+/* vertices_xyz  host, n_vertices x 3 doubles;  tets  host, n_tets x 4 int32 (0-based, any
+ *               orientation);  coeffs  host, n_tets x (k+1)(k+2)(k+3)/6 doubles: coefficients of
+ *               the monomials r^a s^b t^c of the unit reference tetrahedron, point = v0 +
+ *               r (v1 - v0) + s (v2 - v0) + t (v3 - v0), modes ordered by a+b+c, then c, then b.
+ * Errors: SIAC_EINVAL (k outside 1..3, h, domain, (3k+1)h larger than a periodic extent, indices,
+ *   zero-volume tetrahedra, non-finite data), SIAC_EDEVICE, SIAC_ENOMEM, SIAC_ECUDA. */
+siac_status siac3_create(siac3_ctx **out, const double *vertices_xyz, int64_t n_vertices,
+                         const int32_t *tets, int64_t n_tets, const double *coeffs, const siac3_params *params);
+/* host buffers, blocking: points_xyz n_points x 3 -> values_out n_points (input order).  Reports
+ * SIAC_EINTERNAL if a piece stack overflowed (h much smaller than the tetrahedra). */
+siac_status siac3_eval(siac3_ctx *ctx, const double *points_xyz, int64_t n_points, double *values_out);
+/* device buffers, stream-ordered (cuda_stream NULL = legacy default stream). */
+siac_status siac3_eval_async(siac3_ctx *ctx, const double *d_points_xyz, int64_t n_points, double *d_values_out,
+                             void *cuda_stream);
+/* counting of (point, tetrahedron image) pairs and integrated pieces in later evaluations */
+siac_status siac3_set_counting(siac3_ctx *ctx, int32_t enable);
+siac_status siac3_stats(const siac3_ctx *ctx, int64_t *pairs, int64_t *pieces);
+/* host: the collapsed rule on the unit tetrahedron with n^3 points, exact for degree 2n-1:
+ * out n^3 x 4 doubles (r, s, t, weight); weights sum to 1/6. */
+siac_status siac3_tet_rule(int32_t n, double *out);
+void        siac3_destroy(siac3_ctx *ctx);
+const char *siac3_last_error(const siac3_ctx *ctx);
+
 /* Free everything the context owns.  NULL-safe. */
 void siac_destroy(siac_ctx *ctx);
 

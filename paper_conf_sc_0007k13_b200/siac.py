@@ -24,7 +24,8 @@ if os.environ.get("SIAC_LIB_VARIANT"):
     LIB_PATH = os.path.join(_HERE, f"libsiac_b200.{os.environ['SIAC_LIB_VARIANT']}.so")
 SOURCES = [os.path.join(_HERE, "csrc", f) for f in (
     "siac.cu", "siac_eval_k.cu", "siac_internal.h", "siac_device.cuh", "siac_tile.cuh", "siac_ws.cuh",
-    "siac_clipfast.cuh", "siac_jump.cuh", "siac_math.cpp", "siac_math.h", "siac_quadrature.h", "siac_io.cu")]
+    "siac_clipfast.cuh", "siac_jump.cuh", "siac_math.cpp", "siac_math.h", "siac_quadrature.h", "siac_io.cu",
+    "siac3d.cu")]
 SOURCES.append(os.path.join(os.path.dirname(_HERE), "include", "siac.h"))
 
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
@@ -59,6 +60,8 @@ def build(force: bool = False, verbose: bool = False, extra_flags=(), out_path: 
              os.path.join(objdir, "siac_math.o"), cs("siac_math.cpp", "siac_math.h"))]
     jobs.append(([nvcc] + flags + ["-c", "-o", os.path.join(objdir, "siac_io.o")] + cs("siac_io.cu"),
                  os.path.join(objdir, "siac_io.o"), cs("siac_io.cu", "siac_internal.h", "siac_math.h") + [SOURCES[-1]]))
+    jobs.append(([nvcc] + flags + ["-c", "-o", os.path.join(objdir, "siac3d.o")] + cs("siac3d.cu"),
+                 os.path.join(objdir, "siac3d.o"), cs("siac3d.cu", "siac_internal.h", "siac_math.h") + [SOURCES[-1]]))
     jobs.append(([nvcc] + flags + ["-c", "-o", os.path.join(objdir, "siac.o")] + cs("siac.cu"),
                  os.path.join(objdir, "siac.o"), cs("siac.cu", "siac_jump.cuh", "siac_math.h") + common))
     for k in (1, 2, 3, 4):
@@ -114,6 +117,11 @@ class _CreateInfo(ctypes.Structure):
     _fields_ = [("total_ms", ctypes.c_double), ("host_ms", ctypes.c_double), ("h2d_ms", ctypes.c_double),
                 ("index_ms", ctypes.c_double), ("jump_ms", ctypes.c_double), ("cross_ms", ctypes.c_double),
                 ("device_bytes", ctypes.c_int64), ("bytes_per_triangle", ctypes.c_int64)]
+
+
+class _Params3(ctypes.Structure):
+    _fields_ = [("k", ctypes.c_int32), ("h", ctypes.c_double), ("periodic", ctypes.c_int32),
+                ("domain", ctypes.c_double * 6), ("device", ctypes.c_int32)]
 
 
 class _Counters(ctypes.Structure):
@@ -177,6 +185,23 @@ def lib():
         L.siac_project_async.argtypes = [I32, I32, vp, I64, vp, vp]
         L.siac_error_norms_async.restype = ctypes.c_int
         L.siac_error_norms_async.argtypes = [vp, vp, vp, I64, vp, vp]
+        L.siac3_create.restype = ctypes.c_int
+        L.siac3_create.argtypes = [ctypes.POINTER(vp), D, I64, ctypes.POINTER(ctypes.c_int32), I64, D,
+                                   ctypes.POINTER(_Params3)]
+        L.siac3_eval.restype = ctypes.c_int
+        L.siac3_eval.argtypes = [vp, D, I64, D]
+        L.siac3_eval_async.restype = ctypes.c_int
+        L.siac3_eval_async.argtypes = [vp, vp, I64, vp, vp]
+        L.siac3_set_counting.restype = ctypes.c_int
+        L.siac3_set_counting.argtypes = [vp, I32]
+        L.siac3_stats.restype = ctypes.c_int
+        L.siac3_stats.argtypes = [vp, ctypes.POINTER(I64), ctypes.POINTER(I64)]
+        L.siac3_tet_rule.restype = ctypes.c_int
+        L.siac3_tet_rule.argtypes = [I32, D]
+        L.siac3_destroy.restype = None
+        L.siac3_destroy.argtypes = [vp]
+        L.siac3_last_error.restype = ctypes.c_char_p
+        L.siac3_last_error.argtypes = [vp]
         _lib = L
     return _lib
 
@@ -185,7 +210,9 @@ EXPORTED = ["siac_create", "siac_eval", "siac_eval_async", "siac_set_counting", 
             "siac_set_schedule", "siac_set_graphs", "siac_set_timing", "siac_timing", "siac_probe_fp64",
             "siac_info", "siac_host_tables", "siac_debug_records",
             "siac_destroy", "siac_last_error", "siac_version",
-            "siac_projection_rule", "siac_map_points_async", "siac_project_async", "siac_error_norms_async"]
+            "siac_projection_rule", "siac_map_points_async", "siac_project_async", "siac_error_norms_async",
+            "siac3_create", "siac3_eval", "siac3_eval_async", "siac3_set_counting", "siac3_stats", "siac3_tet_rule",
+            "siac3_destroy", "siac3_last_error"]
 
 
 def _dp(a):
@@ -387,3 +414,78 @@ def error_norms_async(d_u, d_ref, d_w, d_out, stream=None) -> None:
     """d_out[0:3] = sqrt(sum w e^2), max |e|, sum w for e = u - ref (d_w may be None)."""
     _check(lib().siac_error_norms_async(_ptr(d_u), _ptr(d_ref), None if d_w is None else _ptr(d_w),
                                         int(d_u.shape[0]), _ptr(d_out), _stream_ptr(stream)), None)
+
+
+# ---------------------------------------------------------------- tetrahedral meshes (NEXT-4)
+
+def _check3(rc, ctx_ptr=None):
+    if rc != 0:
+        raise SiacError(f"siac3 error {rc}: {lib().siac3_last_error(ctx_ptr).decode()}")
+
+
+class Context3:
+    """A siac3_ctx (include/siac.h, tetrahedral meshes): coefficients of the reference-tetrahedron
+    monomials r^a s^b t^c (modes by a+b+c, then c, then b)."""
+
+    def __init__(self, V, T, C, k: int, h: float, periodic: int = 7, domain=(0.0, 0.0, 0.0, 1.0, 1.0, 1.0),
+                 device: int = 0):
+        L = lib()
+        V = np.ascontiguousarray(V, dtype=np.float64).reshape(-1, 3)
+        T = np.ascontiguousarray(T, dtype=np.int32).reshape(-1, 4)
+        C = np.ascontiguousarray(C, dtype=np.float64)
+        if 1 <= k <= 3 and C.size != len(T) * (k + 1) * (k + 2) * (k + 3) // 6:
+            raise ValueError("coeffs must have (k+1)(k+2)(k+3)/6 columns")
+        p = _Params3(int(k), float(h), int(periodic), (ctypes.c_double * 6)(*domain), int(device))
+        ptr = ctypes.c_void_p()
+        _check3(L.siac3_create(ctypes.byref(ptr), _dp(V), len(V), T.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)),
+                               len(T), _dp(C), ctypes.byref(p)), None)
+        self._ptr = ptr
+        self.k = int(k)
+
+    def eval(self, points) -> np.ndarray:
+        P = np.ascontiguousarray(points, dtype=np.float64).reshape(-1, 3)
+        out = np.empty(len(P), dtype=np.float64)
+        _check3(lib().siac3_eval(self._ptr, _dp(P), len(P), _dp(out)), self._ptr)
+        return out
+
+    def eval_async(self, d_points, d_out, stream=None) -> None:
+        assert d_points.dtype.is_floating_point and d_points.element_size() == 8 and d_points.is_contiguous()
+        assert d_out.element_size() == 8 and d_out.is_contiguous()
+        n = d_points.numel() // 3
+        assert d_out.numel() >= n
+        if stream is None:
+            import torch
+            stream = torch.cuda.current_stream(d_points.device)
+        sh = stream.cuda_stream if hasattr(stream, "cuda_stream") else (stream or 0)
+        _check3(lib().siac3_eval_async(self._ptr, ctypes.c_void_p(d_points.data_ptr()), n,
+                                       ctypes.c_void_p(d_out.data_ptr()), ctypes.c_void_p(sh)), self._ptr)
+
+    def set_counting(self, on: bool = True) -> None:
+        _check3(lib().siac3_set_counting(self._ptr, 1 if on else 0), self._ptr)
+
+    def stats(self) -> dict:
+        a, b = ctypes.c_int64(), ctypes.c_int64()
+        _check3(lib().siac3_stats(self._ptr, ctypes.byref(a), ctypes.byref(b)), self._ptr)
+        return {"pairs": a.value, "pieces": b.value}
+
+    def destroy(self) -> None:
+        if getattr(self, "_ptr", None):
+            lib().siac3_destroy(self._ptr)
+            self._ptr = None
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+
+def create3(V, T, C, k, h, periodic=7, domain=(0.0, 0.0, 0.0, 1.0, 1.0, 1.0), device=0) -> Context3:
+    return Context3(V, T, C, k, h, periodic, domain, device)
+
+
+def tet_rule(n: int) -> np.ndarray:
+    """(n^3, 4): (r, s, t, weight) of the library's collapsed rule on the unit tetrahedron."""
+    out = np.empty((n ** 3, 4))
+    _check3(lib().siac3_tet_rule(int(n), _dp(out)), None)
+    return out

@@ -20,7 +20,7 @@ def L():
 
 def _declared():
     txt = open(os.path.join(ROOT, "include", "siac.h")).read()
-    return sorted(set(re.findall(r"^\s*(?:siac_status|void|const char \*)\s*(siac_\w+)\s*\(", txt, re.M)))
+    return sorted(set(re.findall(r"^\s*(?:siac_status|void|const char \*)\s*(siac3?_\w+)\s*\(", txt, re.M)))
 
 
 def test_header_declares_expected_calls():
@@ -115,3 +115,18 @@ def test_host_basis_matrix(L, k):
     mono = np.stack([rho ** a * sig ** b for a, b in order], axis=1)
     ref = inputs.dubiner_eval(k, 2 * r - 1, 2 * s - 1)
     assert np.abs(mono @ R.T - ref).max() < 1e-12
+
+
+def test_tet_rule_exact(L):
+    """siac3_tet_rule (host): the collapsed Gauss-Jacobi rule on the unit tetrahedron integrates
+    r^a s^b t^c exactly up to degree 2n-1: a! b! c! / (a+b+c+3)! (Dirichlet integral)."""
+    from math import factorial
+    for n in (2, 4, 5):
+        q = siac.tet_rule(n)
+        assert q.shape == (n ** 3, 4) and np.all(q[:, 3] > 0)
+        for a in range(2 * n):
+            for b in range(2 * n - a):
+                for c in range(2 * n - a - b):
+                    exact = factorial(a) * factorial(b) * factorial(c) / factorial(a + b + c + 3)
+                    got = np.sum(q[:, 3] * q[:, 0] ** a * q[:, 1] ** b * q[:, 2] ** c)
+                    assert abs(got - exact) < 1e-15 + 1e-13 * exact, (n, a, b, c)
