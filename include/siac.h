@@ -280,7 +280,8 @@ siac_status siac_debug_records(siac_ctx *ctx, int32_t which, int64_t n, double *
  * product of three 1D kernels (L212-214) -- integrated exactly as in Eq. (2): each tetrahedron
  * the stencil touches is cut by the kernel breakplanes into pieces inside single kernel cells
  * (depth-first plane splits; a cut tetrahedron is a tetrahedron + a prism or two prisms, a prism
- * 3 tetrahedra), each piece integrated by a collapsed Gauss-Jacobi rule exact for degree 3k.
+ * 3 tetrahedra), each piece integrated by a collapsed Gauss-Jacobi rule exact for degree 4k
+ * (three kernel factors of degree k and u of degree k).
  * Direct method (thread per point); conventions as for the 2D calls above. */
 typedef struct siac3_ctx siac3_ctx;
 typedef struct {

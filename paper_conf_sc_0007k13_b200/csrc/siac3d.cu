@@ -3,7 +3,7 @@
 // Eq. (1): u*(x) = (1/h^3) \int K((y1-x1)/h) K((y2-x2)/h) K((y3-x3)/h) u_h(y) dy (the stencil is
 // the tensor product of 1D kernels, L212-214), computed exactly as in Eq. (2): every tetrahedron
 // the stencil touches is cut by the kernel breakplanes into pieces inside single kernel cells,
-// and each piece is integrated by a rule exact for the integrand's degree 3k.
+// and each piece is integrated by a rule exact for the integrand's degree 4k (K K K u).
 //
 // B200 design (direct method; the 2D library's spline-jump decomposition is not carried over):
 //   siac3_create: H2D of V, T, modes; k_prep3 (per-tetrahedron record: vertices, inverse affine
@@ -45,7 +45,7 @@ inline void need3(bool ok, const char *msg) {
     if (!ok) throw Fail3{SIAC_EINVAL, std::string(msg)};
 }
 
-constexpr int MAXQ3 = 125;        // quadrature points (k = 3: 5^3)
+constexpr int MAXQ3 = 343;        // quadrature points (k = 3: 7^3)
 constexpr int STACK3 = 64;        // depth-first split stack (tetrahedra); overflow is reported
 
 template <int K> struct Rec3 {
@@ -303,8 +303,10 @@ __global__ void __launch_bounds__(128) k_eval3(Eval3Args a) {
                         for (int d = 0; d < 3 && ax < 0; ++d) {
                             double mn = tt.p[0][d], mx = tt.p[0][d];
                             for (int i = 1; i < 4; ++i) { mn = fmin(mn, tt.p[i][d]); mx = fmax(mx, tt.p[i][d]); }
-                            const double kn = floor(mn - T0) + 1.0 + T0;     // first plane above the minimum
-                            if (kn < mx && kn >= T0 && kn <= -T0) { ax = d; cut = kn; }   // incl. the support ends
+                            // the first kernel plane (t_0 = T0 .. t_NC = -T0, incl. the support ends)
+                            // strictly above the piece's minimum; a plane inside the piece cuts it
+                            const double kn = fmax(floor(mn - T0) + 1.0 + T0, T0);
+                            if (kn < mx && kn <= -T0) { ax = d; cut = kn; }
                         }
                         if (ax < 0) {
                             // one kernel cell: integrate K K K u over the piece (if inside the support)
@@ -577,7 +579,8 @@ siac_status siac3_create(siac3_ctx **out, const double *V, int64_t nv, const int
         }
         const int64_t ncell = (int64_t)c->nc[0] * c->nc[1] * c->nc[2];
         std::vector<double> kc = siac::kernel_cell_table(p->k);
-        const int nqd = (3 * p->k + 2) / 2;                  // exact for degree 2n - 1 >= 3k
+        // the integrand K(z1) K(z2) K(z3) u has total degree 4k: n^3 points, exact for 2n - 1 >= 4k
+        const int nqd = 2 * p->k + 1;
         std::vector<double> q = tet_rule(nqd);
         c->nq = (int)(q.size() / 4);
         CK3(cudaMalloc(&c->d_kc, sizeof(double) * kc.size()));
