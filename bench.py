@@ -37,7 +37,7 @@ def flops_per_subtri(k):
     return NQ[k] * 2 * (nb + 2 * k + 8)
 
 
-# Schedule JUMP (default) computes the same integral through the spline-jump decomposition
+# Schedules JUMP / JUMPX (JUMPX is the default) compute the same integral through the spline-jump decomposition
 # (DESIGN.md §8.2); its algorithmic FP64 flops per unit, counted from the operations the
 # decomposition needs (an FMA counts 2):
 #   per (point, triangle) pair: two cut tests (10 each), two Taylor shifts of the base cell
@@ -46,8 +46,8 @@ def flops_per_subtri(k):
 #     lambda^(K+2) power (K+1 mul) and the accumulate (1 FMA);
 #   per cross sub-triangle (schedule 4): NQ quadrature points x (affine maps 8 FMA, bivariate
 #     Horner NB-1 FMA, product/weight 2 FMA, t^K: K mul) + 20 set-up;
-#   per interval-polynomial cross term (schedule 5, default): 2D Clenshaw over NP = (K+1)(3K+3)
-#     Chebyshev coefficients (1 FMA + 1 add each) + lambda^(2K+2) and the mapping (~2K + 12).
+#   per interval-polynomial cross term (schedule 5, default): a bivariate Horner/Estrin pass over
+#     NP = (K+1)(3K+3) monomial coefficients (1 FMA each) + lambda^(2K+2) and the mapping (~2K + 12).
 def jump_flops(k, pairs, corners, cross_subtris, cross_polys=0):
     nb = (k + 1) * (k + 2) // 2
     ng = (k + 1) * (3 * k + 2) // 2
@@ -55,7 +55,7 @@ def jump_flops(k, pairs, corners, cross_subtris, cross_polys=0):
     f_pair = 20 + 2 * (k * (k + 1) + (k + 1) * (k + 2))
     f_corner = 2 * (ng + 2 * k + 1) + (k + 1)
     f_xsub = NQ[k] * (2 * (nb + 9) + k) + 20
-    f_xpoly = 3 * npoly + 2 * k + 12
+    f_xpoly = 2 * npoly + 2 * k + 12
     return (pairs * f_pair + corners * f_corner + cross_subtris * f_xsub + cross_polys * f_xpoly,
             (f_pair, f_corner, f_xsub, f_xpoly))
 

@@ -282,7 +282,7 @@ siac_status siac_debug_records(siac_ctx *ctx, int32_t which, int64_t n, double *
  * (depth-first plane splits; a cut tetrahedron is a tetrahedron + a prism or two prisms, a prism
  * 3 tetrahedra), each piece integrated by a collapsed Gauss-Jacobi rule exact for degree 4k
  * (three kernel factors of degree k and u of degree k).
- * Direct method (thread per point); conventions as for the 2D calls above. */
+ * Direct method (warp per point tile, siac3_set_schedule); conventions as for the 2D calls above. */
 typedef struct siac3_ctx siac3_ctx;
 typedef struct {
     int32_t k;          /* dG degree 1..3 */
@@ -306,6 +306,12 @@ siac_status siac3_eval(siac3_ctx *ctx, const double *points_xyz, int64_t n_point
 /* device buffers, stream-ordered (cuda_stream NULL = legacy default stream). */
 siac_status siac3_eval_async(siac3_ctx *ctx, const double *d_points_xyz, int64_t n_points, double *d_values_out,
                              void *cuda_stream);
+/* Evaluation mapping for later evaluations (same decomposition, rule and result up to rounding
+ * order): 0 (default) = warp per 32-point tile -- the tile's candidate tetrahedra walked
+ * warp-uniformly, the pieces split per lane and queued in shared memory, the quadrature run 32
+ * pieces at a time in lock step; 1 = thread per point (the paper's per-point mapping, Alg. 2,
+ * PAPER.md L552-565).  SIAC_EINVAL for other values. */
+siac_status siac3_set_schedule(siac3_ctx *ctx, int32_t schedule);
 /* counting of (point, tetrahedron image) pairs and integrated pieces in later evaluations */
 siac_status siac3_set_counting(siac3_ctx *ctx, int32_t enable);
 siac_status siac3_stats(const siac3_ctx *ctx, int64_t *pairs, int64_t *pieces);

@@ -9,12 +9,14 @@
 //   siac3_create: H2D of V, T, modes; k_prep3 (per-tetrahedron record: vertices, inverse affine
 //     map, modes in the reference monomial basis; bounding box; anchor cell = bbox-min cell of a
 //     uniform grid); CUB radix sort by anchor cell; k_gather3; CSR cell_start.
-//   siac3_eval_async: k_point_keys3 (periodic wrap, 30-bit Morton key) + CUB sort -> k_eval3, one
-//     thread per point in Morton order: the cells of the stencil box (extended by the largest
-//     tetrahedron extent), box test per candidate image, then a depth-first stack that splits the
-//     tetrahedron by every kernel plane strictly crossing it (a plane cut yields a tetrahedron
-//     plus a prism, or two prisms; prisms are cut into 3 tetrahedra) until every piece lies in one
-//     kernel cell, and a collapsed Gauss(-Jacobi) rule on each piece; one write per point.
+//   siac3_eval_async: k_point_keys3 (periodic wrap, 30-bit Morton key) + CUB sort -> k_eval3w
+//     (default), one warp per 32-point tile in Morton order: the cells of the tile's stencil box
+//     (extended by the largest tetrahedron extent), box tests per candidate image, then per lane a
+//     depth-first stack that splits the tetrahedron by every kernel plane strictly crossing it (a
+//     plane cut yields a tetrahedron plus a prism, or two prisms; prisms are cut into 3
+//     tetrahedra) until every piece lies in one kernel cell; the pieces are queued in shared
+//     memory and integrated 32 at a time by a collapsed Gauss(-Jacobi) rule; one write per point.
+//     k_eval3 (schedule 1) is the thread-per-point mapping of the same steps.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -177,6 +179,7 @@ struct Eval3Args {
     int periodic;
     double h, inv_h, hw;
     unsigned long long *cnt;  // pairs, pieces
+    int split;                // k_eval3w: warps per point tile (1, 2, 4), each walking a share of the cells
 };
 
 __global__ void k_point_keys3(const double *pts, int64_t np, double x0, double y0, double z0, double Lx, double Ly,
@@ -297,6 +300,13 @@ __global__ void __launch_bounds__(128) k_eval3(Eval3Args a) {
                         for (int d = 0; d < 3; ++d) stack[0].p[i][d] = ((__ldg(rc + 3 * i + d) + sh[d]) - x[d]) * a.inv_h;
                     while (ns > 0) {
                         const Tet tt = stack[--ns];
+                        bool outside = false;             // a piece outside the support on an axis: K = 0, drop
+                        for (int d = 0; d < 3; ++d) {
+                            const double mn = fmin(fmin(tt.p[0][d], tt.p[1][d]), fmin(tt.p[2][d], tt.p[3][d]));
+                            const double mx = fmax(fmax(tt.p[0][d], tt.p[1][d]), fmax(tt.p[2][d], tt.p[3][d]));
+                            outside = outside || mx <= T0 || mn >= -T0;
+                        }
+                        if (outside) continue;
                         // the first kernel plane strictly crossing the piece (axes x, y, z in order)
                         int ax = -1;
                         double cut = 0.0;
@@ -396,6 +406,380 @@ __global__ void __launch_bounds__(128) k_eval3(Eval3Args a) {
         atomicAdd(a.cnt + 0, c_pairs);
         atomicAdd(a.cnt + 1, c_pieces);
     }
+}
+
+// ------------------------------------------------------------------ warp per point tile (default)
+// The same decomposition and rule as k_eval3, mapped for SIMD efficiency: one warp owns a tile of
+// 32 Morton-consecutive points (each point written by exactly one warp: the buffered stencil of
+// PAPER.md L340-347, no races); the candidate tetrahedra of the tile's stencil box are walked
+// warp-uniformly (32 boxes tested per step, ballot); for each candidate the lanes whose stencil
+// meets it split it depth-first (divergent but cheap), and every leaf piece is appended to the
+// warp's shared-memory piece queue; the quadrature -- the dominant cost, (2k+1)^3 points per
+// piece -- runs 32 queued pieces at a time, one per lane, in lock step.  Piece values are added
+// to their owner points in lane order (deterministic).
+constexpr int TW3 = 4;            // warps per block
+constexpr int QC3 = 64;           // piece queue per warp: < 32 left over + <= 32 new
+
+struct PieceQ3 {
+    double p[12][QC3];            // vertex 0 (3) and edges v1-v0, v2-v0, v3-v0 (9), z-units of the owner
+    double r0[3][QC3];            // reference coordinates of the owner's z = 0: Ainv (x - shift - v0)
+    double vol6[QC3];             // 6 |volume| (z-units)
+    int tet[QC3];
+    int info[QC3];                // owner lane | cell x << 5 | cell y << 9 | cell z << 13
+    double acc[32];               // per-owner sums of the flushed pieces
+};
+
+__device__ __forceinline__ unsigned lanemask_lt3() {
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+template <int K>
+__device__ __forceinline__ void flush3(const Eval3Args &a, PieceQ3 &Q, const double *kc, const double *qr, int &nq,
+                                       int lane) {
+    using R = Rec3<K>;
+    constexpr double T0 = -0.5 * (3 * K + 1);
+    const int take = min(nq, 32);
+    int key = 32;                 // no owner
+    double v = 0.0;
+    if (lane < take) {
+        const int e = nq - 1 - lane;
+        const int info = Q.info[e];
+        key = info & 31;
+        const int ci[3] = {(info >> 5) & 15, (info >> 9) & 15, (info >> 13) & 15};
+        const double *rc = a.rec + (int64_t)R::RS * Q.tet[e];
+        double M[9], cf[R::NB];
+#pragma unroll
+        for (int j = 0; j < 9; ++j) M[j] = a.h * __ldg(rc + R::OFF_AINV + j);
+#pragma unroll
+        for (int j = 0; j < R::NB; ++j) cf[j] = __ldg(rc + R::OFF_C + j);
+        // z(xi, eta, zeta) = p0 + xi E0 + eta E1 + zeta E2;  rst = r0 + M z = A + xi B0 + eta B1 + zeta B2;
+        // the kernel factors are evaluated in cell-centred variables (p0 shifted by the cell centre)
+        double pc[3], E[3][3], A[3], B[3][3];
+#pragma unroll
+        for (int d = 0; d < 3; ++d) {
+            pc[d] = Q.p[d][e];
+#pragma unroll
+            for (int j = 0; j < 3; ++j) E[j][d] = Q.p[3 + 3 * j + d][e];
+        }
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+            A[i] = fma(M[3 * i], pc[0], fma(M[3 * i + 1], pc[1], fma(M[3 * i + 2], pc[2], Q.r0[i][e])));
+#pragma unroll
+            for (int j = 0; j < 3; ++j) B[j][i] = fma(M[3 * i], E[j][0], fma(M[3 * i + 1], E[j][1], M[3 * i + 2] * E[j][2]));
+        }
+        double kr[3][K + 1];
+#pragma unroll
+        for (int d = 0; d < 3; ++d) {
+            pc[d] -= T0 + ci[d] + 0.5;
+#pragma unroll
+            for (int j = 0; j <= K; ++j) kr[d][j] = kc[ci[d] * (K + 1) + j];
+        }
+        double s = 0.0;
+        for (int q = 0; q < a.nq; ++q) {
+            const double2 xe = *reinterpret_cast<const double2 *>(qr + 4 * q);
+            const double2 zw = *reinterpret_cast<const double2 *>(qr + 4 * q + 2);
+            double kv = 1.0;
+#pragma unroll
+            for (int d = 0; d < 3; ++d)
+                kv *= horner1<K>(kr[d], fma(zw.x, E[2][d], fma(xe.y, E[1][d], fma(xe.x, E[0][d], pc[d]))));
+            const double rr = fma(zw.x, B[2][0], fma(xe.y, B[1][0], fma(xe.x, B[0][0], A[0])));
+            const double ss = fma(zw.x, B[2][1], fma(xe.y, B[1][1], fma(xe.x, B[0][1], A[1])));
+            const double tt = fma(zw.x, B[2][2], fma(xe.y, B[1][2], fma(xe.x, B[0][2], A[2])));
+            s = fma(zw.y * kv, umono<K>(cf, rr, ss, tt), s);
+        }
+        v = Q.vol6[e] * s;
+    }
+    nq -= take;
+    // per-owner sums in lane order (deterministic): the group leader adds the others' values
+    const unsigned grp = __match_any_sync(0xffffffffu, key);
+    const int leader = __ffs(grp) - 1;
+    double sum = v;
+    unsigned rest = grp & ~(1u << leader);
+    while (__any_sync(0xffffffffu, rest != 0)) {
+        const int src = rest ? __ffs(rest) - 1 : lane;
+        const double w = __shfl_sync(0xffffffffu, v, src);
+        if (rest) { sum += w; rest &= rest - 1; }
+    }
+    if (lane == leader && key < 32) Q.acc[key] += sum;
+    __syncwarp();
+}
+
+template <int K, bool COUNT, int MINB>
+__global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
+    using R = Rec3<K>;
+    constexpr int NC = 3 * K + 1;
+    constexpr double T0 = -0.5 * (3 * K + 1);
+    constexpr int NKC = (NC * (K + 1) + 1) & ~1;
+    extern __shared__ __align__(16) double sm3[];
+    double *kc = sm3;
+    double *qr = kc + NKC;
+    PieceQ3 *qs = reinterpret_cast<PieceQ3 *>(qr + ((4 * a.nq + 1) & ~1));
+    for (int i = threadIdx.x; i < NC * (K + 1); i += blockDim.x) kc[i] = a.kc[i];
+    for (int i = threadIdx.x; i < a.nq * 4; i += blockDim.x) qr[i] = a.qr[i];
+    __syncthreads();
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    PieceQ3 &Q = qs[wid];
+    // a.split warps share one tile (small problems: fewer tiles than resident warps), each walking
+    // a contiguous share of the tile's candidate cells; their sums are combined in a fixed order
+    const int split = a.split, part = wid % split;
+    const int64_t p0 = ((int64_t)blockIdx.x * (TW3 / split) + wid / split) * 32;
+    const bool live = p0 < a.np;
+    if (split == 1 && !live) return;              // warp-uniform; no block barrier below for split == 1
+    const bool valid = live && p0 + lane < a.np;
+    int orig = -1;
+    double x[3] = {0.0, 0.0, 0.0};
+    if (valid) {
+        orig = a.perm[p0 + lane];
+        for (int d = 0; d < 3; ++d) {
+            x[d] = a.pts[3 * (int64_t)orig + d];
+            if (a.periodic & (1 << d)) {
+                x[d] = x[d] - a.L[d] * floor((x[d] - a.x0[d]) / a.L[d]);
+                if (x[d] >= a.x0[d] + a.L[d]) x[d] -= a.L[d];
+                if (x[d] < a.x0[d]) x[d] = a.x0[d];
+            }
+        }
+    }
+    Q.acc[lane] = 0.0;
+    int lo[3], hi[3];
+    double tb0[3], tb1[3];
+#pragma unroll
+    for (int d = 0; d < 3; ++d) {
+        double mn = valid ? x[d] : 1e300, mx = valid ? x[d] : -1e300;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            mn = fmin(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+            mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        }
+        tb0[d] = mn - a.hw;       // the tile's stencil box
+        tb1[d] = mx + a.hw;
+        lo[d] = (int)floor((tb0[d] - a.ext[d] - a.x0[d]) / a.cell[d]) - 1;
+        hi[d] = (int)floor((tb1[d] - a.x0[d]) / a.cell[d]) + 1;
+        if (!(a.periodic & (1 << d))) { lo[d] = max(lo[d], 0); hi[d] = min(hi[d], a.nc[d] - 1); }
+    }
+    __syncwarp();
+    int nq = 0;
+    unsigned long long c_pairs = 0, c_pieces = 0;
+    bool overflow = false;
+    Tet stack[STACK3];
+    const int nx = hi[0] - lo[0] + 1, ny = hi[1] - lo[1] + 1;
+    const int64_t ncl = live ? (int64_t)nx * ny * (hi[2] - lo[2] + 1) : 0;
+    const int64_t cl0 = ncl * part / split, cl1 = ncl * (part + 1) / split;
+    for (int64_t cl = cl0; cl < cl1; ++cl) {
+                const int I[3] = {lo[0] + (int)(cl % nx), lo[1] + (int)((cl / nx) % ny), lo[2] + (int)(cl / ((int64_t)nx * ny))};
+                int cidx[3];
+                double sh[3];
+#pragma unroll
+                for (int d = 0; d < 3; ++d) {
+                    cidx[d] = I[d];
+                    int q = 0;
+                    if (a.periodic & (1 << d)) { cidx[d] = ((I[d] % a.nc[d]) + a.nc[d]) % a.nc[d]; q = (I[d] - cidx[d]) / a.nc[d]; }
+                    sh[d] = q * a.L[d];
+                }
+                const int cell = (cidx[2] * a.nc[1] + cidx[1]) * a.nc[0] + cidx[0];
+                const int t0 = __ldg(a.cell_start + cell), t1 = __ldg(a.cell_start + cell + 1);
+                for (int tb = t0; tb < t1; tb += 32) {
+                    bool keep = false;
+                    if (tb + lane < t1) {
+                        const double *bb = a.bbox + 6 * (int64_t)(tb + lane);
+                        keep = true;
+#pragma unroll
+                        for (int d = 0; d < 3; ++d)
+                            keep = keep && (__ldg(bb + d) + sh[d] < tb1[d]) && (__ldg(bb + 3 + d) + sh[d] > tb0[d]);
+                    }
+                    unsigned km = __ballot_sync(0xffffffffu, keep);
+                    while (km) {
+                        const int t = tb + __ffs(km) - 1;
+                        km &= km - 1;
+                        const double *bb = a.bbox + 6 * (int64_t)t;
+                        bool hit = valid;
+#pragma unroll
+                        for (int d = 0; d < 3; ++d)
+                            hit = hit && (__ldg(bb + d) + sh[d] < x[d] + a.hw) && (__ldg(bb + 3 + d) + sh[d] > x[d] - a.hw);
+                        if (!__any_sync(0xffffffffu, hit)) continue;
+                        if (COUNT) c_pairs += hit;
+                        const double *rc = a.rec + (int64_t)R::RS * t;
+                        int ns = 0;
+                        bool have = false;        // tt holds a piece to process (the pair's tetrahedron first)
+                        Tet tt;
+                        double r0[3] = {0.0, 0.0, 0.0};
+                        if (hit) {
+                            double d0[3];
+#pragma unroll
+                            for (int d = 0; d < 3; ++d) d0[d] = x[d] - sh[d] - __ldg(rc + d);
+#pragma unroll
+                            for (int i = 0; i < 3; ++i)
+#pragma unroll
+                                for (int j = 0; j < 3; ++j) r0[i] = fma(__ldg(rc + R::OFF_AINV + 3 * i + j), d0[j], r0[i]);
+                            for (int i = 0; i < 4; ++i)
+                                for (int d = 0; d < 3; ++d) tt.p[i][d] = ((__ldg(rc + 3 * i + d) + sh[d]) - x[d]) * a.inv_h;
+                            have = true;
+                        }
+                        while (__any_sync(0xffffffffu, have || ns > 0)) {
+                            bool leaf = false;
+                            double vol6 = 0.0;
+                            int ci[3] = {0, 0, 0};
+                            if (!have && ns > 0) { tt = stack[--ns]; have = true; }
+                            if (have) {
+                                have = false;
+                                double mn[3], mx[3];
+                                bool outside = false;
+#pragma unroll
+                                for (int d = 0; d < 3; ++d) {
+                                    mn[d] = fmin(fmin(tt.p[0][d], tt.p[1][d]), fmin(tt.p[2][d], tt.p[3][d]));
+                                    mx[d] = fmax(fmax(tt.p[0][d], tt.p[1][d]), fmax(tt.p[2][d], tt.p[3][d]));
+                                    outside = outside || mx[d] <= T0 || mn[d] >= -T0;   // K = 0 there: drop
+                                }
+                                int ax = -1;
+                                double cut = 0.0;
+#pragma unroll
+                                for (int d = 2; d >= 0; --d) {      // the first axis (x, y, z order) cut by a kernel plane
+                                    const double kn = fmax(floor(mn[d] - T0) + 1.0 + T0, T0);
+                                    if (kn < mx[d] && kn <= -T0) { ax = d; cut = kn; }
+                                }
+                                if (outside) {
+                                } else if (ax < 0) {
+                                    // the centroid's cell; a piece whose centroid lies outside the
+                                    // support is dropped (a plane within rounding of its lower end is
+                                    // not found by the search above, e.g. [2 - 1e-16, 2.5] at k = 1)
+                                    bool inside = true;
+                                    for (int d = 0; d < 3; ++d) {
+                                        const double cen = 0.25 * (tt.p[0][d] + tt.p[1][d] + tt.p[2][d] + tt.p[3][d]);
+                                        ci[d] = (int)floor(cen - T0);
+                                        inside = inside && ci[d] >= 0 && ci[d] < NC;
+                                    }
+                                    double e[3][3];
+                                    for (int j = 0; j < 3; ++j)
+                                        for (int d = 0; d < 3; ++d) e[j][d] = tt.p[j + 1][d] - tt.p[0][d];
+                                    vol6 = fabs(e[0][0] * (e[1][1] * e[2][2] - e[1][2] * e[2][1]) -
+                                                e[0][1] * (e[1][0] * e[2][2] - e[1][2] * e[2][0]) +
+                                                e[0][2] * (e[1][0] * e[2][1] - e[1][1] * e[2][0]));
+                                    leaf = inside && vol6 > 0.0;
+                                } else {
+                                    // children are emitted in order; all but the last go to the stack,
+                                    // the last is processed next (tail iteration, one push/pop less)
+                                    Tet pend;
+                                    bool haspend = false;
+                                    const Tet src = tt;
+                                    int lowi[4], highi[4], nl = 0, nh = 0;
+                                    for (int i = 0; i < 4; ++i) {
+                                        if (src.p[i][ax] <= cut) lowi[nl++] = i;
+                                        else highi[nh++] = i;
+                                    }
+                                    auto isect = [&](int i, int j, double *o) {
+                                        const double r = (cut - src.p[i][ax]) / (src.p[j][ax] - src.p[i][ax]);
+                                        for (int d = 0; d < 3; ++d) o[d] = fma(r, src.p[j][d] - src.p[i][d], src.p[i][d]);
+                                        o[ax] = cut;
+                                    };
+                                    auto push = [&](const double *q0, const double *q1, const double *q2, const double *q3) {
+                                        if (haspend) {
+                                            if (ns >= STACK3) overflow = true;
+                                            else stack[ns++] = pend;
+                                        }
+                                        for (int d = 0; d < 3; ++d) {
+                                            pend.p[0][d] = q0[d]; pend.p[1][d] = q1[d];
+                                            pend.p[2][d] = q2[d]; pend.p[3][d] = q3[d];
+                                        }
+                                        haspend = true;
+                                    };
+                                    auto push_prism = [&](const double *a0, const double *a1, const double *a2,
+                                                          const double *b0, const double *b1, const double *b2) {
+                                        push(a0, a1, a2, b2);
+                                        push(a0, a1, b1, b2);
+                                        push(a0, b0, b1, b2);
+                                    };
+                                    if (nl == 1 || nh == 1) {
+                                        const int o = nl == 1 ? lowi[0] : highi[0];
+                                        const int *rest = nl == 1 ? highi : lowi;
+                                        double q[3][3];
+                                        for (int j = 0; j < 3; ++j) isect(o, rest[j], q[j]);
+                                        push(src.p[o], q[0], q[1], q[2]);
+                                        push_prism(q[0], q[1], q[2], src.p[rest[0]], src.p[rest[1]], src.p[rest[2]]);
+                                    } else {
+                                        const int l0 = lowi[0], l1 = lowi[1], h0 = highi[0], h1 = highi[1];
+                                        double q00[3], q01[3], q10[3], q11[3];
+                                        isect(l0, h0, q00); isect(l0, h1, q01); isect(l1, h0, q10); isect(l1, h1, q11);
+                                        push_prism(src.p[l0], q00, q01, src.p[l1], q10, q11);
+                                        push_prism(src.p[h0], q00, q10, src.p[h1], q01, q11);
+                                    }
+                                    tt = pend;
+                                    have = true;
+                                }
+                            }
+                            const unsigned lm = __ballot_sync(0xffffffffu, leaf);
+                            if (leaf) {
+                                const int pos = nq + __popc(lm & lanemask_lt3());
+#pragma unroll
+                                for (int d = 0; d < 3; ++d) {
+                                    Q.p[d][pos] = tt.p[0][d];
+#pragma unroll
+                                    for (int j = 0; j < 3; ++j) Q.p[3 + 3 * j + d][pos] = tt.p[j + 1][d] - tt.p[0][d];
+                                    Q.r0[d][pos] = r0[d];
+                                }
+                                Q.vol6[pos] = vol6;
+                                Q.tet[pos] = t;
+                                Q.info[pos] = lane | (ci[0] << 5) | (ci[1] << 9) | (ci[2] << 13);
+                            }
+                            nq += __popc(lm);
+                            if (COUNT) c_pieces += leaf;
+                            if (nq >= 32) {
+                                __syncwarp();
+                                flush3<K>(a, Q, kc, qr, nq, lane);
+                            }
+                        }
+                    }
+                }
+            }
+    while (nq > 0) {
+        __syncwarp();
+        flush3<K>(a, Q, kc, qr, nq, lane);
+    }
+    __syncwarp();
+    if (split == 1) {
+        if (valid) a.out[orig] = Q.acc[lane];
+    } else {
+        __syncthreads();
+        if (part == 0 && valid) {
+            double v = Q.acc[lane];
+            for (int q = 1; q < split; ++q) v += qs[wid + q].acc[lane];
+            a.out[orig] = v;
+        }
+    }
+    if (__any_sync(0xffffffffu, overflow) && lane == 0) atomicOr(a.cnt + 2, 1ull);
+    if (COUNT) {
+        atomicAdd(a.cnt + 0, c_pairs);
+        atomicAdd(a.cnt + 1, c_pieces);
+    }
+}
+
+// Launch k_eval3w: when the point tiles do not fill one wave of resident warps, each tile's cells
+// are split over 2 or 4 warps (a.split) so that more warps share the work.
+template <int K, bool COUNT, int MINB>
+void launch3w_mb(int64_t ntiles, int num_sms, size_t sm, cudaStream_t st, Eval3Args a) {
+    auto kern = k_eval3w<K, COUNT, MINB>;
+    CK3(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    int per_sm = 0;
+    CK3(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * TW3, sm));
+    const int64_t resident = (int64_t)std::max(per_sm, 1) * num_sms * TW3;
+    a.split = 1;
+    while (a.split < TW3 && ntiles * a.split * 2 <= resident) a.split *= 2;
+    const int tpb = TW3 / a.split;
+    kern<<<(unsigned)((ntiles + tpb - 1) / tpb), 32 * TW3, sm, st>>>(a);
+}
+template <int K, bool COUNT>
+void launch3w(int minb, int64_t ntiles, int num_sms, size_t sm, cudaStream_t st, const Eval3Args &a) {
+    // measured (tools/gpu_s3c.sh): 3 blocks/SM (168 registers) is faster at k = 1 (the splitting
+    // dominates), the unbounded variant at k = 2, 3 (the quadrature's registers)
+    if (minb == 0) minb = K == 1 ? 3 : 1;
+    if (minb >= 4) launch3w_mb<K, COUNT, 4>(ntiles, num_sms, sm, st, a);
+    else if (minb == 3) launch3w_mb<K, COUNT, 3>(ntiles, num_sms, sm, st, a);
+    else launch3w_mb<K, COUNT, 1>(ntiles, num_sms, sm, st, a);
+}
+
+inline size_t smem3w(int k, int nq) {
+    const int nc = 3 * k + 1;
+    return sizeof(double) * (((nc * (k + 1) + 1) & ~1) + ((4 * nq + 1) & ~1)) + TW3 * sizeof(PieceQ3);
 }
 
 // Gauss-Jacobi rule for the weight (1-x)^alpha on [-1, 1] (Golub-Welsch, Jacobi eigenvalue
@@ -507,6 +891,9 @@ struct siac3_ctx {
     int64_t cap_h = 0;
     unsigned long long *d_cnt = nullptr;
     bool counting = false;
+    int schedule = 0;         // 0: warp per point tile (k_eval3w, default), 1: thread per point (k_eval3)
+    int num_sms = 148;
+    int minb = 0;             // k_eval3w __launch_bounds__ min blocks; 0 = per degree (env SIAC3_MINB: experiments)
     std::string err;
 };
 
@@ -550,7 +937,11 @@ siac_status siac3_create(siac3_ctx **out, const double *V, int64_t nv, const int
         CK3(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, p->device));
         if (major < 10) throw Fail3{SIAC_EDEVICE, "device is not sm_100 class"};
         CK3(cudaSetDevice(p->device));
+        int nsm = 0;
+        CK3(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device));
         c = new siac3_ctx();
+        c->num_sms = nsm;
+        if (const char *e = getenv("SIAC3_MINB")) c->minb = atoi(e);
         c->device = p->device;
         c->k = p->k;
         c->h = p->h;
@@ -707,14 +1098,22 @@ siac_status siac3_eval_async(siac3_ctx *ctx, const double *d_pts, int64_t np, do
         a.cnt = ctx->d_cnt;
         if (ctx->counting) CK3(cudaMemsetAsync(ctx->d_cnt, 0, 2 * sizeof(unsigned long long), st));
         const unsigned grid = nblk3(np, 128);
+        const int64_t ntiles = (np + 31) / 32;
+        a.split = 1;
         if (ctx->nt == 0) {
             CK3(cudaMemsetAsync(d_out, 0, sizeof(double) * np, st));
             return;
         }
-#define SIAC3_LAUNCH(KK)                                                                 \
-    do {                                                                                 \
-        if (ctx->counting) k_eval3<KK, true><<<grid, 128, 0, st>>>(a);                  \
-        else k_eval3<KK, false><<<grid, 128, 0, st>>>(a);                               \
+#define SIAC3_LAUNCH(KK)                                                                       \
+    do {                                                                                       \
+        if (ctx->schedule == 1) {                                                              \
+            if (ctx->counting) k_eval3<KK, true><<<grid, 128, 0, st>>>(a);                    \
+            else k_eval3<KK, false><<<grid, 128, 0, st>>>(a);                                 \
+        } else {                                                                               \
+            const size_t sm = smem3w(KK, a.nq);                                                \
+            if (ctx->counting) launch3w<KK, true>(ctx->minb, ntiles, ctx->num_sms, sm, st, a); \
+            else launch3w<KK, false>(ctx->minb, ntiles, ctx->num_sms, sm, st, a);              \
+        }                                                                                      \
     } while (0)
         if (ctx->k == 1) SIAC3_LAUNCH(1);
         else if (ctx->k == 2) SIAC3_LAUNCH(2);
@@ -752,6 +1151,13 @@ siac_status siac3_eval(siac3_ctx *ctx, const double *pts, int64_t np, double *ou
         CK3(cudaStreamSynchronize(ctx->stream));
         if (ovf) throw Fail3{SIAC_EINTERNAL, "piece stack overflow (h much smaller than the tetrahedra)"};
     });
+}
+
+siac_status siac3_set_schedule(siac3_ctx *ctx, int32_t schedule) {
+    if (!ctx) { g_err3 = "NULL context"; return SIAC_EINVAL; }
+    if (schedule < 0 || schedule > 1) { ctx->err = "schedule must be 0 (warp per point tile) or 1 (thread per point)"; return SIAC_EINVAL; }
+    ctx->schedule = schedule;
+    return SIAC_OK;
 }
 
 siac_status siac3_set_counting(siac3_ctx *ctx, int32_t enable) {

@@ -373,9 +373,6 @@ __global__ void k_prep_cross(const double *jrec, int64_t nt, double *xrec, const
 #define SIAC_JUMP_PREFETCH 2      // candidates ahead whose hot record lines are prefetched into L1
 #endif
 constexpr int WARPS = SIAC_JUMP_WARPS;
-#ifndef SIAC_JUMP_CUNIF
-#define SIAC_JUMP_CUNIF 0         // experiment: uncut lanes read their quarter-warp leader's corner block
-#endif
 constexpr int QCAP = 64;      // cross-term queue: < 32 left over + <= 32 new
 constexpr int SCAP = 96;      // staged cross sub-triangles: < 32 left over + <= 64 new
 
@@ -1227,16 +1224,7 @@ __global__ void __launch_bounds__(WARPS * 32, XP ? SIAC_JUMPX_MINB : SIAC_JUMP_M
         double am;
         if constexpr (OS) am = os_alpha<K>(a, &osm->c[ux ? 0 : 1][0][lane], mm);
         else am = alpha[mm];
-        int sd = ux ? sdd : 2 + sdd;
-#if SIAC_JUMP_CUNIF
-        // a lane with no knot on either axis (lam = 0: its corner term is 0) reads the corner
-        // block of its quarter-warp's first lane, so each quarter-warp's loads of the staged
-        // record touch fewer distinct blocks (fewer shared-memory wavefronts)
-        {
-            const int sd0 = __shfl_sync(0xffffffffu, sd, lane & ~7);
-            if (!ux && !uy) sd = sd0;
-        }
-#endif
+        const int sd = ux ? sdd : 2 + sdd;
         const double sg = sdd == 0 ? am : -am;
         double cc[K + 1];
 #pragma unroll

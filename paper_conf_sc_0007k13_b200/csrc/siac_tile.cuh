@@ -1,4 +1,4 @@
-// siac_tile.cuh -- the warp-per-point-tile evaluation kernel (schedule "tile", the default).
+// siac_tile.cuh -- the warp-per-point-tile evaluation kernel (schedule TILE: the direct clip-and-integrate method; the default is JUMPX, siac_jump.cuh).
 //
 // One warp owns a tile of 32 Morton-consecutive evaluation points (buffered stencil:
 // every point is written by exactly one warp, so no write races).

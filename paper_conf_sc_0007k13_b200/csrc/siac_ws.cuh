@@ -1,4 +1,4 @@
-// siac_ws.cuh -- warp-specialized evaluation kernel (schedule "ws", the default).
+// siac_ws.cuh -- warp-specialized evaluation kernel (schedule WS: the direct method with producer/consumer warps; the default is JUMPX, siac_jump.cuh).
 //
 // The SIAC sum for a point is a stream of fan sub-triangles whose geometry (candidate
 // search, Sutherland-Hodgman clipping, Alg. 1 / L369-407) is divergent, branchy

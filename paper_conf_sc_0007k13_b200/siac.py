@@ -192,6 +192,8 @@ def lib():
         L.siac3_eval.argtypes = [vp, D, I64, D]
         L.siac3_eval_async.restype = ctypes.c_int
         L.siac3_eval_async.argtypes = [vp, vp, I64, vp, vp]
+        L.siac3_set_schedule.restype = ctypes.c_int
+        L.siac3_set_schedule.argtypes = [vp, I32]
         L.siac3_set_counting.restype = ctypes.c_int
         L.siac3_set_counting.argtypes = [vp, I32]
         L.siac3_stats.restype = ctypes.c_int
@@ -211,7 +213,7 @@ EXPORTED = ["siac_create", "siac_eval", "siac_eval_async", "siac_set_counting", 
             "siac_info", "siac_host_tables", "siac_debug_records",
             "siac_destroy", "siac_last_error", "siac_version",
             "siac_projection_rule", "siac_map_points_async", "siac_project_async", "siac_error_norms_async",
-            "siac3_create", "siac3_eval", "siac3_eval_async", "siac3_set_counting", "siac3_stats", "siac3_tet_rule",
+            "siac3_create", "siac3_eval", "siac3_eval_async", "siac3_set_schedule", "siac3_set_counting", "siac3_stats", "siac3_tet_rule",
             "siac3_destroy", "siac3_last_error"]
 
 
@@ -459,6 +461,10 @@ class Context3:
         sh = stream.cuda_stream if hasattr(stream, "cuda_stream") else (stream or 0)
         _check3(lib().siac3_eval_async(self._ptr, ctypes.c_void_p(d_points.data_ptr()), n,
                                        ctypes.c_void_p(d_out.data_ptr()), ctypes.c_void_p(sh)), self._ptr)
+
+    def set_schedule(self, schedule: int) -> None:
+        """0: warp per point tile (default), 1: thread per point."""
+        _check3(lib().siac3_set_schedule(self._ptr, int(schedule)), self._ptr)
 
     def set_counting(self, on: bool = True) -> None:
         _check3(lib().siac3_set_counting(self._ptr, 1 if on else 0), self._ptr)

@@ -112,3 +112,42 @@ def test_async_and_counters(siac_mod):
     ctx.destroy()
     assert np.array_equal(o.cpu().numpy(), ref)
     assert st["pieces"] >= st["pairs"] > 0
+
+
+@pytest.mark.parametrize("k", [1, 2, 3])
+def test_schedules_agree(siac_mod, oracle_mod, k):
+    """Warp-per-tile (schedule 0, default) and thread-per-point (schedule 1) mappings of the same
+    decomposition: equal to rounding, equal pair and piece counts, both at oracle parity
+    (ragged last tile: the point count is not a multiple of 32).  k = 3 on the structured mesh with
+    h = the tetrahedron extent (W = 10h covers most of the period: a few points only)."""
+    if k < 3:
+        V, T = m3.lattice_delaunay_mesh3({1: 1500, 2: 1200}[k], seed=40 + k)
+        h = _h(V, T, k)
+        P = m3.eval_points3(V, T)[:: {1: 5, 2: 11}[k]][:-3]
+    else:
+        V, T = m3.structured_mesh3(11)
+        h = 1.0 / 11
+        P = m3.eval_points3(V, T)[np.random.default_rng(43).choice(4 * len(T), 9, replace=False)]
+    C = m3.random_modes3(len(T), k, seed=50 + k)
+    vals, stats = [], []
+    for sch in (0, 1):
+        ctx = siac_mod.create3(V, T, C, k, h)
+        ctx.set_schedule(sch)
+        ctx.set_counting(True)
+        vals.append(ctx.eval(P))
+        stats.append(ctx.stats())
+        ctx.destroy()
+    assert stats[0] == stats[1], stats
+    sc = np.abs(vals[1]).max()
+    assert np.abs(vals[0] - vals[1]).max() <= 1e-13 * sc
+    o = oracle_mod.oracle_eval3(V, T, C, k, h, P[:: max(1, len(P) // 16)])
+    assert_parity(vals[0][:: max(1, len(P) // 16)], o)
+
+
+def test_schedule_rejects_unknown(siac_mod):
+    V, T = m3.structured_mesh3(2)
+    C = m3.random_modes3(len(T), 1, seed=1)
+    ctx = siac_mod.create3(V, T, C, 1, 0.2)
+    with pytest.raises(Exception):
+        ctx.set_schedule(2)
+    ctx.destroy()

@@ -4,7 +4,9 @@ resident in HBM, CUDA events; W >= 3 warm-ups), its geometry counts, a model FP6
 parity against the 3D oracle on a sample.  Not the driver's bench (the north_star metric is
 2D); results go to profiles/.
 
-usage: python tools/bench3d.py [ntet] [k] [steps] [oracle_points] [out.json]
+Both mappings are timed: schedule 0 (warp per point tile, default) and 1 (thread per point).
+
+usage: python tools/bench3d.py [ntet] [k] [steps] [oracle_points] [out.json] [time_schedule_1]
 """
 import json
 import os
@@ -30,6 +32,7 @@ def main():
     steps = int(sys.argv[3]) if len(sys.argv) > 3 else 5
     nor = int(sys.argv[4]) if len(sys.argv) > 4 else 24
     out_path = sys.argv[5] if len(sys.argv) > 5 else None
+    tpp = int(sys.argv[6]) if len(sys.argv) > 6 else 1      # also time schedule 1 (thread per point)
     V, T = m3.lattice_delaunay_mesh3(ntet, seed=4000 + k)
     C = m3.project3(V, T, k, m3.sin3)
     h = min(m3.max_extent3(V, T), 0.95 / (3 * k + 1))     # W = (3k+1)h must fit the period
@@ -39,21 +42,26 @@ def main():
     create_ms = 1e3 * (time.perf_counter() - t0)
     d = torch.from_numpy(P).cuda()
     o = torch.empty(len(P), dtype=torch.float64, device="cuda")
-    ctx.set_counting(True)
-    ctx.eval_async(d, o)
-    st = ctx.stats()
-    ctx.set_counting(False)
-    for _ in range(3):
+
+    def timed(schedule):
+        ctx.set_schedule(schedule)
+        ctx.set_counting(True)
         ctx.eval_async(d, o)
-    torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    for _ in range(steps):
-        ctx.eval_async(d, o)
-    e1.record()
-    torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1) / steps
-    g = o.cpu().numpy()
+        st = ctx.stats()
+        ctx.set_counting(False)
+        for _ in range(3):
+            ctx.eval_async(d, o)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(steps):
+            ctx.eval_async(d, o)
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / steps, st, o.cpu().numpy()
+
+    ms, st, g = timed(0)             # warp per point tile (default)
+    ms1, st1, g1 = timed(1) if tpp else (None, None, None)   # thread per point (the paper's per-point mapping)
     ctx.destroy()
     nq = (2 * k + 1) ** 3
     nb = m3.n_modes3(k)
@@ -69,7 +77,12 @@ def main():
     ot = time.perf_counter() - t0
     res = {"what": "NEXT-4 tetrahedral path (siac3_eval_async), FP64", "n_tets": int(len(T)), "n_points": int(len(P)),
            "k": k, "h": h, "mesh": "jittered-lattice Delaunay (scipy), periodic unit cube", "field": "sin sin sin, L2",
+           "schedule": "0: warp per 32-point tile, pieces queued in shared memory, quadrature in lock step",
            "ms_per_eval": ms, "points_per_s": len(P) / (ms * 1e-3), "create_ms": create_ms,
+           "thread_per_point": None if not tpp else {"schedule": 1, "ms_per_eval": ms1, "points_per_s": len(P) / (ms1 * 1e-3),
+                                "model_frac_of_fp64_peak": flops / (ms1 * 1e-3) / peak,
+                                "same_counts": st1 == st,
+                                "max_rel_diff_vs_schedule0": float(np.abs(g1 - g).max() / np.abs(g).max())},
            "pairs": st["pairs"], "pieces": st["pieces"], "pairs_per_point": st["pairs"] / len(P),
            "pieces_per_pair": st["pieces"] / max(st["pairs"], 1), "quadrature_points_per_piece": nq,
            "model_flops_per_eval": flops, "model_tflops": flops / (ms * 1e-3) / 1e12,
