@@ -769,9 +769,10 @@ void launch3w_mb(int64_t ntiles, int num_sms, size_t sm, cudaStream_t st, Eval3A
 }
 template <int K, bool COUNT>
 void launch3w(int minb, int64_t ntiles, int num_sms, size_t sm, cudaStream_t st, const Eval3Args &a) {
-    // measured (tools/gpu_s3c.sh): 3 blocks/SM (168 registers) is faster at k = 1 (the splitting
-    // dominates), the unbounded variant at k = 2, 3 (the quadrature's registers)
-    if (minb == 0) minb = K == 1 ? 3 : 1;
+    // measured (tools/gpu_s3c.sh, gpu_s3e.sh): 4 blocks/SM (128 registers) is faster at k = 1 (the
+    // latency-bound splitting dominates: 821 vs 981 ms at 3 blocks), the unbounded variant at k = 2, 3
+    // (the quadrature's registers: 5.6 s unbounded vs 6.4 s at 3 blocks/SM, k = 2)
+    if (minb == 0) minb = K == 1 ? 4 : 1;
     if (minb >= 4) launch3w_mb<K, COUNT, 4>(ntiles, num_sms, sm, st, a);
     else if (minb == 3) launch3w_mb<K, COUNT, 3>(ntiles, num_sms, sm, st, a);
     else launch3w_mb<K, COUNT, 1>(ntiles, num_sms, sm, st, a);
