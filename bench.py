@@ -445,6 +445,7 @@ def run_siac(args):
                 ncu_rec["file"] = "profiles/" + tp
                 traffic = ncu_rec["bytes_per_point"] * n_local
                 break
+        alg_bytes = 28 * n_local + len(T) * cinfo["bytes_per_triangle"]
         cfgd = workload_desc(w, args.config)
         cfgd.update({"parallelism": f"spatial point tiles x{world} + halo, NCCL all_gather" if world > 1
                      else "single GPU",
@@ -463,8 +464,11 @@ def run_siac(args):
                 "roofline": {"bound": "alu", "kernel": "k_eval", "achieved": achieved, "peak": peak,
                              "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,
                              "traffic_note": ("dram read+write bytes per launch from the committed ncu --set full "
-                                              "capture (%s), scaled by this launch's points; algorithmic ~41 B/point"
-                                              % (ncu_rec["file"] if ncu_rec else "none")),
+                                              "capture (%s), scaled by this launch's points" % (ncu_rec["file"] if ncu_rec else "none")),
+                             # compulsory bytes of one launch: points (16 B) + permutation (4 B) + values (8 B)
+                             # per point, and every resident triangle record read at least once
+                             "algorithmic_bytes": alg_bytes,
+                             "traffic_over_algorithmic": (traffic / alg_bytes) if traffic else None,
                              "peak_note": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1965 MHz (DESIGN.md §8.1)",
                              "measured_dfma_peak": peak_meas,
                              "frac_of_measured": (achieved / peak_meas) if achieved else None,
