@@ -417,6 +417,19 @@ __global__ void __launch_bounds__(128) k_eval3(Eval3Args a) {
 // warp's shared-memory piece queue; the quadrature -- the dominant cost, (2k+1)^3 points per
 // piece -- runs 32 queued pieces at a time, one per lane, in lock step.  Piece values are added
 // to their owner points in lane order (deterministic).
+// Device-side bounds checks (debug builds: -DSIAC_DEVICE_CHECKS=1, e.g. tools/build_variant.py);
+// a failed check prints its condition and traps.
+#ifndef SIAC_DEVICE_CHECKS
+#define SIAC_DEVICE_CHECKS 0
+#endif
+#define CHK3(c)                                                                                   \
+    do {                                                                                          \
+        if (SIAC_DEVICE_CHECKS && !(c)) {                                                         \
+            printf("siac3d device check failed: %s (line %d)\n", #c, __LINE__);                   \
+            __trap();                                                                             \
+        }                                                                                         \
+    } while (0)
+
 constexpr int TW3 = 4;            // warps per block
 constexpr int QC3 = 64;           // piece queue per warp: < 32 left over + <= 32 new
 
@@ -445,9 +458,11 @@ __device__ __forceinline__ void flush3(const Eval3Args &a, PieceQ3 &Q, const dou
     double v = 0.0;
     if (lane < take) {
         const int e = nq - 1 - lane;
+        CHK3(e >= 0 && e < QC3);
         const int info = Q.info[e];
         key = info & 31;
         const int ci[3] = {(info >> 5) & 15, (info >> 9) & 15, (info >> 13) & 15};
+        CHK3(ci[0] < 3 * K + 1 && ci[1] < 3 * K + 1 && ci[2] < 3 * K + 1 && Q.tet[e] >= 0);
         const double *rc = a.rec + (int64_t)R::RS * Q.tet[e];
         double M[9], cf[R::NB];
 #pragma unroll
@@ -564,7 +579,8 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
     bool overflow = false;
     Tet stack[STACK3];
     const int nx = hi[0] - lo[0] + 1, ny = hi[1] - lo[1] + 1;
-    const int64_t ncl = live ? (int64_t)nx * ny * (hi[2] - lo[2] + 1) : 0;
+    const int nz = hi[2] - lo[2] + 1;             // (empty when a non-periodic axis clamps the range away)
+    const int64_t ncl = (live && nx > 0 && ny > 0 && nz > 0) ? (int64_t)nx * ny * nz : 0;
     const int64_t cl0 = ncl * part / split, cl1 = ncl * (part + 1) / split;
     for (int64_t cl = cl0; cl < cl1; ++cl) {
                 const int I[3] = {lo[0] + (int)(cl % nx), lo[1] + (int)((cl / nx) % ny), lo[2] + (int)(cl / ((int64_t)nx * ny))};
@@ -578,6 +594,7 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
                     sh[d] = q * a.L[d];
                 }
                 const int cell = (cidx[2] * a.nc[1] + cidx[1]) * a.nc[0] + cidx[0];
+                CHK3(cidx[0] >= 0 && cidx[0] < a.nc[0] && cidx[1] >= 0 && cidx[1] < a.nc[1] && cidx[2] >= 0 && cidx[2] < a.nc[2]);
                 const int t0 = __ldg(a.cell_start + cell), t1 = __ldg(a.cell_start + cell + 1);
                 for (int tb = t0; tb < t1; tb += 32) {
                     bool keep = false;
@@ -689,27 +706,35 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
                                         push(a0, a1, b1, b2);
                                         push(a0, b0, b1, b2);
                                     };
+                                    // a side beyond a support end plane (cut = T0: the low side, cut =
+                                    // -T0: the high side) is outside the support: not emitted (k >= 2;
+                                    // at k = 1 the extra registers cost more than the saved pushes:
+                                    // A/B on one box, tools/gpu_ab3.sh: k = 1 878 vs 822 ms, k = 2 5266
+                                    // vs 5611 ms; the outside pieces are dropped when popped instead)
+                                    const bool keep_lo = K == 1 || cut > T0, keep_hi = K == 1 || cut < -T0;
                                     if (nl == 1 || nh == 1) {
                                         const int o = nl == 1 ? lowi[0] : highi[0];
                                         const int *rest = nl == 1 ? highi : lowi;
                                         double q[3][3];
                                         for (int j = 0; j < 3; ++j) isect(o, rest[j], q[j]);
-                                        push(src.p[o], q[0], q[1], q[2]);
-                                        push_prism(q[0], q[1], q[2], src.p[rest[0]], src.p[rest[1]], src.p[rest[2]]);
+                                        if (nl == 1 ? keep_lo : keep_hi) push(src.p[o], q[0], q[1], q[2]);
+                                        if (nl == 1 ? keep_hi : keep_lo)
+                                            push_prism(q[0], q[1], q[2], src.p[rest[0]], src.p[rest[1]], src.p[rest[2]]);
                                     } else {
                                         const int l0 = lowi[0], l1 = lowi[1], h0 = highi[0], h1 = highi[1];
                                         double q00[3], q01[3], q10[3], q11[3];
                                         isect(l0, h0, q00); isect(l0, h1, q01); isect(l1, h0, q10); isect(l1, h1, q11);
-                                        push_prism(src.p[l0], q00, q01, src.p[l1], q10, q11);
-                                        push_prism(src.p[h0], q00, q10, src.p[h1], q01, q11);
+                                        if (keep_lo) push_prism(src.p[l0], q00, q01, src.p[l1], q10, q11);
+                                        if (keep_hi) push_prism(src.p[h0], q00, q10, src.p[h1], q01, q11);
                                     }
                                     tt = pend;
-                                    have = true;
+                                    have = haspend;
                                 }
                             }
                             const unsigned lm = __ballot_sync(0xffffffffu, leaf);
                             if (leaf) {
                                 const int pos = nq + __popc(lm & lanemask_lt3());
+                                CHK3(pos < QC3 && ci[0] >= 0 && ci[0] < NC && ci[1] >= 0 && ci[1] < NC && ci[2] >= 0 && ci[2] < NC);
 #pragma unroll
                                 for (int d = 0; d < 3; ++d) {
                                     Q.p[d][pos] = tt.p[0][d];
@@ -742,7 +767,10 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
         __syncthreads();
         if (part == 0 && valid) {
             double v = Q.acc[lane];
-            for (int q = 1; q < split; ++q) v += qs[wid + q].acc[lane];
+            for (int q = 1; q < split; ++q) {
+                CHK3(wid + q < TW3);
+                v += qs[wid + q].acc[lane];
+            }
             a.out[orig] = v;
         }
     }

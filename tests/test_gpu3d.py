@@ -151,3 +151,21 @@ def test_schedule_rejects_unknown(siac_mod):
     with pytest.raises(Exception):
         ctx.set_schedule(2)
     ctx.destroy()
+
+
+def test_points_outside_nonperiodic_domain(siac_mod, oracle_mod):
+    """Zero extension on non-periodic axes: whole point tiles far outside the domain (empty
+    candidate-cell ranges after clamping) give exactly 0; mixed tiles match the oracle."""
+    V, T = m3.structured_mesh3(4)
+    C = m3.random_modes3(len(T), 1, seed=61)
+    rng = np.random.default_rng(62)
+    far = rng.uniform(-9, -3, (40, 3))
+    near = rng.uniform(-0.3, 1.3, (30, 3))
+    P = np.concatenate([far, near])
+    for sch in (0, 1):
+        ctx = siac_mod.create3(V, T, C, 1, 0.2, periodic=0)
+        ctx.set_schedule(sch)
+        g = ctx.eval(P)
+        ctx.destroy()
+        assert np.all(g[:40] == 0.0)
+        assert_parity(g[40:], oracle_mod.oracle_eval3(V, T, C, 1, 0.2, near, periodic=0))
