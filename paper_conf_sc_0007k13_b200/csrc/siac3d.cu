@@ -442,6 +442,16 @@ struct PieceQ3 {
     double acc[32];               // per-owner sums of the flushed pieces
 };
 
+// Pending pieces of the current candidate tetrahedron shared by the warp's lanes: a lane that has
+// finished its own pair takes pieces split off by the others (the split work is balanced across the
+// warp; a lane's own overflow goes to its local-memory stack).
+constexpr int WQ3 = 64;
+struct WorkQ3 {
+    double p[12][WQ3];            // the 4 vertices (z-units of the owner point)
+    int owner[WQ3];               // owner lane
+    double r0[3][32];             // per owner lane: reference coordinates of its z = 0 (this candidate)
+};
+
 __device__ __forceinline__ unsigned lanemask_lt3() {
     unsigned m;
     asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -536,6 +546,7 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
     __syncthreads();
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     PieceQ3 &Q = qs[wid];
+    WorkQ3 &W = reinterpret_cast<WorkQ3 *>(qs + TW3)[wid];
     // a.split warps share one tile (small problems: fewer tiles than resident warps), each walking
     // a contiguous share of the tile's candidate cells; their sums are combined in a fixed order
     const int split = a.split, part = wid % split;
@@ -578,6 +589,7 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
     unsigned long long c_pairs = 0, c_pieces = 0;
     bool overflow = false;
     Tet stack[STACK3];
+    int stack_own[STACK3];
     const int nx = hi[0] - lo[0] + 1, ny = hi[1] - lo[1] + 1;
     const int nz = hi[2] - lo[2] + 1;             // (empty when a non-periodic axis clamps the range away)
     const int64_t ncl = (live && nx > 0 && ny > 0 && nz > 0) ? (int64_t)nx * ny * nz : 0;
@@ -617,27 +629,52 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
                         if (!__any_sync(0xffffffffu, hit)) continue;
                         if (COUNT) c_pairs += hit;
                         const double *rc = a.rec + (int64_t)R::RS * t;
-                        int ns = 0;
+                        int ns = 0, wn = 0;       // local stack depth; shared work-queue length (warp-uniform)
                         bool have = false;        // tt holds a piece to process (the pair's tetrahedron first)
+                        int own = lane;           // owner lane of tt
                         Tet tt;
-                        double r0[3] = {0.0, 0.0, 0.0};
+                        __syncwarp();             // the previous candidate's leaves have read W.r0
                         if (hit) {
                             double d0[3];
 #pragma unroll
                             for (int d = 0; d < 3; ++d) d0[d] = x[d] - sh[d] - __ldg(rc + d);
 #pragma unroll
-                            for (int i = 0; i < 3; ++i)
+                            for (int i = 0; i < 3; ++i) {
+                                double r = 0.0;
 #pragma unroll
-                                for (int j = 0; j < 3; ++j) r0[i] = fma(__ldg(rc + R::OFF_AINV + 3 * i + j), d0[j], r0[i]);
+                                for (int j = 0; j < 3; ++j) r = fma(__ldg(rc + R::OFF_AINV + 3 * i + j), d0[j], r);
+                                W.r0[i][lane] = r;
+                            }
                             for (int i = 0; i < 4; ++i)
                                 for (int d = 0; d < 3; ++d) tt.p[i][d] = ((__ldg(rc + 3 * i + d) + sh[d]) - x[d]) * a.inv_h;
                             have = true;
                         }
-                        while (__any_sync(0xffffffffu, have || ns > 0)) {
+                        while (true) {
+                            // refill: own local stack first, then idle lanes take pieces of the shared queue
+                            if (!have && ns > 0) { --ns; tt = stack[ns]; own = stack_own[ns]; have = true; }
+                            const unsigned idle = __ballot_sync(0xffffffffu, !have);
+                            const int take = min(__popc(idle), wn);
+                            if (!have) {
+                                const int rk = __popc(idle & lanemask_lt3());
+                                if (rk < take) {
+                                    const int e = wn - 1 - rk;
+#pragma unroll
+                                    for (int i = 0; i < 4; ++i)
+#pragma unroll
+                                        for (int d = 0; d < 3; ++d) tt.p[i][d] = W.p[3 * i + d][e];
+                                    own = W.owner[e];
+                                    have = true;
+                                }
+                            }
+                            wn -= take;
+                            if (!__any_sync(0xffffffffu, have)) break;
+                            __syncwarp();         // slots [wn, wn + take) are read before they are refilled
                             bool leaf = false;
                             double vol6 = 0.0;
                             int ci[3] = {0, 0, 0};
-                            if (!have && ns > 0) { tt = stack[--ns]; have = true; }
+                            bool split = false;
+                            int ax = -1, npush = 0;
+                            double cut = 0.0;
                             if (have) {
                                 have = false;
                                 double mn[3], mx[3];
@@ -648,8 +685,6 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
                                     mx[d] = fmax(fmax(tt.p[0][d], tt.p[1][d]), fmax(tt.p[2][d], tt.p[3][d]));
                                     outside = outside || mx[d] <= T0 || mn[d] >= -T0;   // K = 0 there: drop
                                 }
-                                int ax = -1;
-                                double cut = 0.0;
 #pragma unroll
                                 for (int d = 2; d >= 0; --d) {      // the first axis (x, y, z order) cut by a kernel plane
                                     const double kn = fmax(floor(mn[d] - T0) + 1.0 + T0, T0);
@@ -674,62 +709,96 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
                                                 e[0][2] * (e[1][0] * e[2][1] - e[1][1] * e[2][0]));
                                     leaf = inside && vol6 > 0.0;
                                 } else {
-                                    // children are emitted in order; all but the last go to the stack,
-                                    // the last is processed next (tail iteration, one push/pop less)
-                                    Tet pend;
-                                    bool haspend = false;
-                                    const Tet src = tt;
-                                    int lowi[4], highi[4], nl = 0, nh = 0;
-                                    for (int i = 0; i < 4; ++i) {
-                                        if (src.p[i][ax] <= cut) lowi[nl++] = i;
-                                        else highi[nh++] = i;
-                                    }
-                                    auto isect = [&](int i, int j, double *o) {
-                                        const double r = (cut - src.p[i][ax]) / (src.p[j][ax] - src.p[i][ax]);
-                                        for (int d = 0; d < 3; ++d) o[d] = fma(r, src.p[j][d] - src.p[i][d], src.p[i][d]);
-                                        o[ax] = cut;
-                                    };
-                                    auto push = [&](const double *q0, const double *q1, const double *q2, const double *q3) {
-                                        if (haspend) {
-                                            if (ns >= STACK3) overflow = true;
-                                            else stack[ns++] = pend;
-                                        }
-                                        for (int d = 0; d < 3; ++d) {
-                                            pend.p[0][d] = q0[d]; pend.p[1][d] = q1[d];
-                                            pend.p[2][d] = q2[d]; pend.p[3][d] = q3[d];
-                                        }
-                                        haspend = true;
-                                    };
-                                    auto push_prism = [&](const double *a0, const double *a1, const double *a2,
-                                                          const double *b0, const double *b1, const double *b2) {
-                                        push(a0, a1, a2, b2);
-                                        push(a0, a1, b1, b2);
-                                        push(a0, b0, b1, b2);
-                                    };
+                                    split = true;
+                                    int nl = 0;
+                                    for (int i = 0; i < 4; ++i) nl += tt.p[i][ax] <= cut;
                                     // a side beyond a support end plane (cut = T0: the low side, cut =
-                                    // -T0: the high side) is outside the support: not emitted (k >= 2;
-                                    // at k = 1 the extra registers cost more than the saved pushes:
-                                    // A/B on one box, tools/gpu_ab3.sh: k = 1 878 vs 822 ms, k = 2 5266
-                                    // vs 5611 ms; the outside pieces are dropped when popped instead)
-                                    const bool keep_lo = K == 1 || cut > T0, keep_hi = K == 1 || cut < -T0;
-                                    if (nl == 1 || nh == 1) {
-                                        const int o = nl == 1 ? lowi[0] : highi[0];
-                                        const int *rest = nl == 1 ? highi : lowi;
-                                        double q[3][3];
-                                        for (int j = 0; j < 3; ++j) isect(o, rest[j], q[j]);
-                                        if (nl == 1 ? keep_lo : keep_hi) push(src.p[o], q[0], q[1], q[2]);
-                                        if (nl == 1 ? keep_hi : keep_lo)
-                                            push_prism(q[0], q[1], q[2], src.p[rest[0]], src.p[rest[1]], src.p[rest[2]]);
-                                    } else {
-                                        const int l0 = lowi[0], l1 = lowi[1], h0 = highi[0], h1 = highi[1];
-                                        double q00[3], q01[3], q10[3], q11[3];
-                                        isect(l0, h0, q00); isect(l0, h1, q01); isect(l1, h0, q10); isect(l1, h1, q11);
-                                        if (keep_lo) push_prism(src.p[l0], q00, q01, src.p[l1], q10, q11);
-                                        if (keep_hi) push_prism(src.p[h0], q00, q10, src.p[h1], q01, q11);
-                                    }
-                                    tt = pend;
-                                    have = haspend;
+                                    // -T0: the high side) is outside the support: not emitted
+                                    const int nlo = cut > T0 ? (nl == 1 ? 1 : 3) : 0;      // tets on the low side
+                                    const int nhi = cut < -T0 ? (nl == 3 ? 1 : 3) : 0;     // (2-2: 3 and 3)
+                                    npush = nlo + nhi - 1;                                // all but the last child
                                 }
+                            }
+                            // children go to the shared queue while it has room (a prefix of the lanes),
+                            // the rest to their lanes' local stacks
+                            int excl = npush;
+#pragma unroll
+                            for (int o = 1; o < 32; o <<= 1) {
+                                const int v = __shfl_up_sync(0xffffffffu, excl, o);
+                                if (lane >= o) excl += v;
+                            }
+                            excl -= npush;
+                            const bool fits = wn + excl + npush <= WQ3;
+                            const int pushed = __reduce_add_sync(0xffffffffu, (split && fits) ? npush : 0);
+                            if (split) {
+                                Tet pend;
+                                bool haspend = false;
+                                int slot = wn + excl;
+                                const Tet src = tt;
+                                int lowi[4], highi[4], nl = 0, nh = 0;
+                                for (int i = 0; i < 4; ++i) {
+                                    if (src.p[i][ax] <= cut) lowi[nl++] = i;
+                                    else highi[nh++] = i;
+                                }
+                                auto isect = [&](int i, int j, double *o) {
+                                    const double r = (cut - src.p[i][ax]) / (src.p[j][ax] - src.p[i][ax]);
+                                    for (int d = 0; d < 3; ++d) o[d] = fma(r, src.p[j][d] - src.p[i][d], src.p[i][d]);
+                                    o[ax] = cut;
+                                };
+                                auto push = [&](const double *q0, const double *q1, const double *q2, const double *q3) {
+                                    if (haspend) {
+                                        if (fits) {
+                                            CHK3(slot < WQ3);
+#pragma unroll
+                                            for (int i = 0; i < 4; ++i)
+#pragma unroll
+                                                for (int d = 0; d < 3; ++d) W.p[3 * i + d][slot] = pend.p[i][d];
+                                            W.owner[slot] = own;
+                                            ++slot;
+                                        } else if (ns >= STACK3) {
+                                            overflow = true;
+                                        } else {
+                                            stack[ns] = pend;
+                                            stack_own[ns] = own;
+                                            ++ns;
+                                        }
+                                    }
+                                    for (int d = 0; d < 3; ++d) {
+                                        pend.p[0][d] = q0[d]; pend.p[1][d] = q1[d];
+                                        pend.p[2][d] = q2[d]; pend.p[3][d] = q3[d];
+                                    }
+                                    haspend = true;
+                                };
+                                auto push_prism = [&](const double *a0, const double *a1, const double *a2,
+                                                      const double *b0, const double *b1, const double *b2) {
+                                    push(a0, a1, a2, b2);
+                                    push(a0, a1, b1, b2);
+                                    push(a0, b0, b1, b2);
+                                };
+                                const bool keep_lo = cut > T0, keep_hi = cut < -T0;
+                                if (nl == 1 || nh == 1) {
+                                    const int o = nl == 1 ? lowi[0] : highi[0];
+                                    const int *rest = nl == 1 ? highi : lowi;
+                                    double q[3][3];
+                                    for (int j = 0; j < 3; ++j) isect(o, rest[j], q[j]);
+                                    if (nl == 1 ? keep_lo : keep_hi) push(src.p[o], q[0], q[1], q[2]);
+                                    if (nl == 1 ? keep_hi : keep_lo)
+                                        push_prism(q[0], q[1], q[2], src.p[rest[0]], src.p[rest[1]], src.p[rest[2]]);
+                                } else {
+                                    const int l0 = lowi[0], l1 = lowi[1], h0 = highi[0], h1 = highi[1];
+                                    double q00[3], q01[3], q10[3], q11[3];
+                                    isect(l0, h0, q00); isect(l0, h1, q01); isect(l1, h0, q10); isect(l1, h1, q11);
+                                    if (keep_lo) push_prism(src.p[l0], q00, q01, src.p[l1], q10, q11);
+                                    if (keep_hi) push_prism(src.p[h0], q00, q10, src.p[h1], q01, q11);
+                                }
+                                tt = pend;
+                                have = haspend;
+                            }
+                            wn += pushed;
+                            double r0[3] = {0.0, 0.0, 0.0};
+                            if (leaf) {
+#pragma unroll
+                                for (int d = 0; d < 3; ++d) r0[d] = W.r0[d][own];
                             }
                             const unsigned lm = __ballot_sync(0xffffffffu, leaf);
                             if (leaf) {
@@ -744,7 +813,7 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
                                 }
                                 Q.vol6[pos] = vol6;
                                 Q.tet[pos] = t;
-                                Q.info[pos] = lane | (ci[0] << 5) | (ci[1] << 9) | (ci[2] << 13);
+                                Q.info[pos] = own | (ci[0] << 5) | (ci[1] << 9) | (ci[2] << 13);
                             }
                             nq += __popc(lm);
                             if (COUNT) c_pieces += leaf;
@@ -797,10 +866,10 @@ void launch3w_mb(int64_t ntiles, int num_sms, size_t sm, cudaStream_t st, Eval3A
 }
 template <int K, bool COUNT>
 void launch3w(int minb, int64_t ntiles, int num_sms, size_t sm, cudaStream_t st, const Eval3Args &a) {
-    // measured (tools/gpu_s3c.sh, gpu_s3e.sh): 4 blocks/SM (128 registers) is faster at k = 1 (the
-    // latency-bound splitting dominates: 821 vs 981 ms at 3 blocks), the unbounded variant at k = 2, 3
-    // (the quadrature's registers: 5.6 s unbounded vs 6.4 s at 3 blocks/SM, k = 2)
-    if (minb == 0) minb = K == 1 ? 4 : 1;
+    // measured (tools/gpu_wq3.sh, with the shared work queue): 3 blocks/SM (168 registers) at k = 1
+    // (709 vs 739 ms at 4 blocks), the unbounded variant at k = 2, 3 (the quadrature's registers:
+    // 5.6 s unbounded vs 6.4 s at 3 blocks/SM, k = 2, before the work queue)
+    if (minb == 0) minb = K == 1 ? 3 : 1;
     if (minb >= 4) launch3w_mb<K, COUNT, 4>(ntiles, num_sms, sm, st, a);
     else if (minb == 3) launch3w_mb<K, COUNT, 3>(ntiles, num_sms, sm, st, a);
     else launch3w_mb<K, COUNT, 1>(ntiles, num_sms, sm, st, a);
@@ -808,7 +877,7 @@ void launch3w(int minb, int64_t ntiles, int num_sms, size_t sm, cudaStream_t st,
 
 inline size_t smem3w(int k, int nq) {
     const int nc = 3 * k + 1;
-    return sizeof(double) * (((nc * (k + 1) + 1) & ~1) + ((4 * nq + 1) & ~1)) + TW3 * sizeof(PieceQ3);
+    return sizeof(double) * (((nc * (k + 1) + 1) & ~1) + ((4 * nq + 1) & ~1)) + TW3 * (sizeof(PieceQ3) + sizeof(WorkQ3));
 }
 
 // Gauss-Jacobi rule for the weight (1-x)^alpha on [-1, 1] (Golub-Welsch, Jacobi eigenvalue
