@@ -654,21 +654,24 @@ __global__ void __launch_bounds__(TW3 * 32, MINB) k_eval3w(Eval3Args a) {
                             if (!have && ns > 0) { --ns; tt = stack[ns]; own = stack_own[ns]; have = true; }
                             const unsigned idle = __ballot_sync(0xffffffffu, !have);
                             const int take = min(__popc(idle), wn);
-                            if (!have) {
-                                const int rk = __popc(idle & lanemask_lt3());
-                                if (rk < take) {
-                                    const int e = wn - 1 - rk;
+                            if (take > 0) {                   // warp-uniform
+                                __syncwarp();                 // W (pieces, owners' r0) written by other lanes is visible
+                                if (!have) {
+                                    const int rk = __popc(idle & lanemask_lt3());
+                                    if (rk < take) {
+                                        const int e = wn - 1 - rk;
 #pragma unroll
-                                    for (int i = 0; i < 4; ++i)
+                                        for (int i = 0; i < 4; ++i)
 #pragma unroll
-                                        for (int d = 0; d < 3; ++d) tt.p[i][d] = W.p[3 * i + d][e];
-                                    own = W.owner[e];
-                                    have = true;
+                                            for (int d = 0; d < 3; ++d) tt.p[i][d] = W.p[3 * i + d][e];
+                                        own = W.owner[e];
+                                        have = true;
+                                    }
                                 }
+                                __syncwarp();                 // slots [wn - take, wn) are read before they are refilled
                             }
                             wn -= take;
                             if (!__any_sync(0xffffffffu, have)) break;
-                            __syncwarp();         // slots [wn, wn + take) are read before they are refilled
                             bool leaf = false;
                             double vol6 = 0.0;
                             int ci[3] = {0, 0, 0};
