@@ -979,7 +979,10 @@ __device__ __forceinline__ void cross_stage(const JumpArgs &a, SM_ &S, XQueue &Q
 }
 
 #ifndef SIAC_JUMPX_MINB
-#define SIAC_JUMPX_MINB SIAC_JUMP_MINB
+// 5 blocks/SM (102 registers, small spills) for the default schedule: A/B on one box, 2 reps
+// (profiles/r02g_ab_2d_minb5.txt): cfg 5 349.8 vs 354.4 ms, cfg 4 61.1 vs 62.0 ms, cfg 3 12.97
+// vs 12.6 ms -- the large problems gain, the small graded one loses a little
+#define SIAC_JUMPX_MINB 5
 #endif
 // OS (one-sided kernels near non-periodic boundaries, with XP only): every lane evaluates its own
 // kernel Kt(. - lambda) at the effective point x + lambda h; cell rows and knot jumps are built
