@@ -438,7 +438,7 @@ def run_siac(args):
         # DRAM traffic per launch from the committed ncu --set full capture of this kernel at
         # the bench's own cfg-5 launch (profiles/*_ncu_traffic_cfg5.json), scaled by points
         traffic, ncu_rec = None, None
-        for tp in ("r02b_ncu_traffic_cfg5.json", "r02_ncu_traffic_cfg5.json", "r01_ncu_traffic_jumpx.json"):
+        for tp in ("r02g_ncu_traffic_cfg5.json", "r02b_ncu_traffic_cfg5.json", "r02_ncu_traffic_cfg5.json", "r01_ncu_traffic_jumpx.json"):
             tpath = os.path.join(ROOT, "profiles", tp)
             if args.schedule in (0, 5) and os.path.exists(tpath):
                 ncu_rec = json.load(open(tpath))
