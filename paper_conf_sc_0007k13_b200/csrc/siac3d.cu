@@ -864,6 +864,7 @@ void launch3w_mb(int64_t ntiles, int num_sms, size_t sm, cudaStream_t st, Eval3A
     const int64_t resident = (int64_t)std::max(per_sm, 1) * num_sms * TW3;
     a.split = 1;
     while (a.split < TW3 && ntiles * a.split * 2 <= resident) a.split *= 2;
+    if (const char *e = getenv("SIAC3_SPLIT")) a.split = std::max(1, std::min(TW3, atoi(e)));   // (experiments)
     const int tpb = TW3 / a.split;
     kern<<<(unsigned)((ntiles + tpb - 1) / tpb), 32 * TW3, sm, st>>>(a);
 }
